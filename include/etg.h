@@ -1,0 +1,153 @@
+/*
+ * etg.h -- C ABI of the B200-native EtaGraph frontier-expansion library (libetg.so).
+ *
+ * What it computes (Sec. II-C): "Graph traversal is to calculate
+ * labels of all nodes reachable from a given root node."  Procedure 1 (L205-207):
+ * Data = graph in CSR format, Result = vertex labels, computed by push expansion
+ * of an active set (Def. 1), each active vertex cut into shadow vertices of
+ * at most K out-edges (Unified Degree Cut, Def. 3), neighbour segments
+ * staged in shared memory (SMP, Sec. V-B), labels relaxed with an
+ * atomic min and the next active set compacted (L136-140, L217).
+ *
+ * Conventions (DESIGN.md readings):
+ *   - vertex ids, labels, depths, distances and weights are uint32;
+ *   - INF = 0xFFFFFFFF marks "unreached" (BFS, SSSP); SSSP distances saturate at
+ *     CAP = 0xFFFFFFFE (R-9); n must be <= 0xFFFFFFFE;
+ *   - CSR: row offsets off[n+1] (uint32, or uint64 with ETG_OFFSETS_U64),
+ *     column ids col[m], weights w[m] (structure of arrays, L55).
+ *
+ * Ownership: every d_* pointer is caller-owned DEVICE memory that the library
+ * borrows; the CSR arrays and the workspace must outlive the handle.  Output
+ * arrays are fully overwritten (n entries).  Apart from the handle itself (host
+ * memory) and one small pinned host word, the library allocates nothing, except
+ * in etg_run_host, which works on host buffers.
+ *
+ * Streams: all work is enqueued on the handle's stream (a cudaStream_t passed as
+ * void*, NULL = legacy default stream).  Traversal calls return after the work
+ * has completed (they read back the iteration statistics).  A handle is not
+ * thread-safe; separate handles are independent.
+ *
+ * Errors: functions return a negative etg_status on failure; nothing partial is
+ * guaranteed then.  etg_last_error() returns a thread-local detail string.
+ *
+ * Results never depend on K, ETG_NO_UDC, ETG_NO_SMP or ETG_HOST_LOOP
+ * (Theorems 1-2, L119-127): the labels are unique fixpoints.
+ */
+#ifndef ETG_H
+#define ETG_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct etg_graph etg_graph; /* opaque handle */
+
+typedef enum {
+    ETG_OK = 0,
+    ETG_EINVAL = -1,      /* bad argument (NULL pointer, source >= n, K = 0 with UDC, ...) */
+    ETG_ENOMEM = -2,      /* workspace too small, or host allocation failed */
+    ETG_ECUDA = -3,       /* a CUDA runtime error (detail in etg_last_error) */
+    ETG_ENCCL = -4,       /* reserved for the multi-GPU exchange */
+    ETG_ENOTSYM = -5,     /* etg_cc on a handle loaded without ETG_SYMMETRIC */
+    ETG_ERANGE = -6,      /* sizes exceed the index types (n > 2^32-2, m >= 2^32 with u32 offsets, ...) */
+    ETG_ENOWEIGHTS = -7,  /* etg_sssp / etg_sswp on a handle loaded without weights */
+    ETG_EINVALID_CSR = -8 /* ETG_VALIDATE found a malformed CSR */
+} etg_status;
+
+enum {
+    ETG_SYMMETRIC = 1u << 0,   /* caller asserts the CSR is symmetric (required by etg_cc) */
+    ETG_NO_UDC = 1u << 1,      /* ablation: one work item per active vertex (K = infinity) */
+    ETG_NO_SMP = 1u << 2,      /* ablation: no shared-memory staging of neighbour segments */
+    ETG_OFFSETS_U64 = 1u << 3, /* d_row_offsets holds uint64 (needed when m >= 2^32) */
+    ETG_VALIDATE = 1u << 4,    /* etg_load_csr runs an O(n+m) device check of the CSR */
+    ETG_HOST_LOOP = 1u << 5    /* drive iterations from the host (count read back each
+                                  iteration) instead of a CUDA-graph conditional while node */
+};
+
+typedef struct {
+    uint32_t degree_limit_k; /* K of Def. 3; 0 -> default 32 */
+    uint32_t flags;          /* ETG_* bits above */
+} etg_options;
+
+typedef struct {
+    uint32_t iterations;       /* non-empty active sets processed (Proc. 1 while-loop trips) */
+    uint32_t reserved;
+    uint64_t activations;      /* label improvements that won the atomic (incl. degree-0 vertices) */
+    uint64_t shadows;          /* shadow vertices processed, summed over iterations (|N|, L152) */
+    uint64_t edges_processed;  /* edges relaxed, summed over iterations */
+    uint64_t vertices_reached; /* filled by etg_reach_stats */
+    uint64_t edges_reached;    /* filled by etg_reach_stats: sum of out-degrees of reached vertices */
+    float ms;                  /* device time of the traversal call (CUDA events) */
+} etg_stats;
+
+/* Bytes of device workspace etg_load_csr needs for n vertices and m edges. */
+size_t etg_workspace_bytes(uint64_t n, uint64_t m, const etg_options *opt);
+
+/* Create a handle over a caller-owned device CSR (Proc. 1 "Load data", L207;
+ * the CSR is used unmodified, L113).  d_weights may be NULL (then SSSP/SSWP
+ * return ETG_ENOWEIGHTS).  stream is a cudaStream_t (void* here). */
+etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m,
+                        const void *d_row_offsets, const uint32_t *d_col_idx,
+                        const uint32_t *d_weights, void *d_workspace,
+                        size_t workspace_bytes, void *stream, const etg_options *opt);
+
+/* BFS (Proc. 1 Kernel BFS, L207): d_depth[v] = hop distance from source, INF if
+ * unreachable. */
+etg_status etg_bfs(etg_graph *g, uint32_t source, uint32_t *d_depth, etg_stats *st_or_null);
+
+/* SSSP (L62, L78): d_dist[v] = saturating shortest-path distance (CAP), INF if
+ * unreachable. */
+etg_status etg_sssp(etg_graph *g, uint32_t source, uint32_t *d_dist, etg_stats *st_or_null);
+
+/* CC (BASELINE.json north_star; R-12): d_label[v] = minimum vertex id of v's
+ * connected component.  Requires a handle loaded with ETG_SYMMETRIC. */
+etg_status etg_cc(etg_graph *g, uint32_t *d_label, etg_stats *st_or_null);
+
+/* SSWP (L62, L249; NEXT-1): d_width[v] = max over paths of the minimum edge
+ * weight; width[source] = INF, unreachable = 0. */
+etg_status etg_sswp(etg_graph *g, uint32_t source, uint32_t *d_width, etg_stats *st_or_null);
+
+/* Reach statistics of a label array: vertices with label != unreached and the
+ * sum of their out-degrees (m of the activatable subgraph, Def. 2). */
+etg_status etg_reach_stats(etg_graph *g, const uint32_t *d_label, uint32_t unreached,
+                           etg_stats *st);
+
+/* Step A2 exposed for testing: the Unified Degree Cut of an active set, computed
+ * by the same device code the traversal uses (Def. 3; Sec. IV-A).
+ * d_active[n_active] (device) is the active set; every entry must have
+ * out-degree >= 1 (degree-0 vertices produce no shadow and are filtered before
+ * they reach the active set, L142).  Writes shadow q of the j-th active vertex
+ * in active-set order as (d_id, d_start, d_end) = (v, off[v]+qK,
+ * min(off[v]+(q+1)K, off[v+1])), uint32/uint64/uint64 device arrays of `cap`
+ * entries; *n_out receives the number of shadows (ETG_ENOMEM if > cap). */
+etg_status etg_udc_slices(etg_graph *g, const uint32_t *d_active, uint32_t n_active,
+                          uint32_t *d_id, uint64_t *d_start, uint64_t *d_end,
+                          uint64_t cap, uint64_t *n_out);
+
+/* Release a handle (does not free the borrowed device memory). */
+void etg_free(etg_graph *g);
+
+/* End-to-end entry on HOST buffers (the paper's "total time", L247: transfer +
+ * execution).  alg: 0 = BFS, 1 = SSSP, 2 = CC, 3 = SSWP.  Copies the CSR
+ * host->device into d_scratch (caller-owned device memory of at least
+ * etg_host_scratch_bytes), runs the traversal and copies the n labels back into
+ * h_labels.  Host buffers should be pinned for full PCIe bandwidth. */
+size_t etg_host_scratch_bytes(uint64_t n, uint64_t m, int has_weights, const etg_options *opt);
+etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_row_offsets,
+                        const uint32_t *h_col_idx, const uint32_t *h_weights,
+                        uint32_t source, uint32_t *h_labels, void *d_scratch,
+                        size_t scratch_bytes, void *stream, const etg_options *opt,
+                        etg_stats *st_or_null);
+
+const char *etg_status_str(etg_status s);
+const char *etg_last_error(void);
+/* Number of CUDA kernels this library launched since load (for bench claims). */
+uint64_t etg_kernel_launches(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ETG_H */

@@ -1,0 +1,560 @@
+// etg.cu -- host engine and C ABI of libetg.so (see include/etg.h).
+//
+// The engine owns nothing on the device: the CSR and a caller-provided
+// workspace are borrowed (etg_load_csr).  Per traversal call it enqueues, on the
+// handle's stream: ctl_begin + init (A1), then the Proc. 1 while-loop
+// as a CUDA graph with a conditional WHILE node whose body is
+// udc_scan -> expand -> advance (A2-A6).  The loop condition is set on the
+// device, so the host synchronises once per call, not once per iteration.
+// ETG_HOST_LOOP replaces the graph by a host loop that reads the active-set
+// size back every iteration (the paper's own control flow).
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "../../include/etg.h"
+#include "etg_kernels.cuh"
+
+using namespace etg;
+
+namespace {
+
+thread_local std::string g_err;
+std::atomic<uint64_t> g_launches{0};
+
+etg_status fail(etg_status s, const std::string &msg) {
+    g_err = msg;
+    return s;
+}
+
+#define ETG_CU(call)                                                                          \
+    do {                                                                                      \
+        cudaError_t e_ = (call);                                                              \
+        if (e_ != cudaSuccess) {                                                              \
+            return fail(ETG_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_));     \
+        }                                                                                     \
+    } while (0)
+
+constexpr size_t kAlign = 256;
+size_t align_up(size_t x) { return (x + kAlign - 1) & ~(kAlign - 1); }
+
+struct Params {
+    uint32_t K;
+    uint32_t ts;
+    uint32_t ts_log2;
+    bool udc;
+    bool smp;
+    bool u64;
+};
+
+Params derive(const etg_options *opt) {
+    Params p;
+    const uint32_t flags = opt ? opt->flags : 0u;
+    p.K = (opt && opt->degree_limit_k) ? opt->degree_limit_k : 32u;
+    p.udc = !(flags & ETG_NO_UDC);
+    p.u64 = (flags & ETG_OFFSETS_U64) != 0;
+    // tile of ts shadows; SMP stages at most ts*K words (the UDC bound, L199)
+    constexpr uint32_t kCapE = 8192;
+    p.ts = kBlock;
+    if (p.udc && p.K > kCapE / kBlock) {
+        uint32_t ts = kBlock;
+        while (ts > 32 && ts * (uint64_t)p.K > kCapE) ts >>= 1;
+        p.ts = ts;
+    }
+    p.smp = p.udc && !(flags & ETG_NO_SMP) && (uint64_t)p.ts * p.K <= kCapE;
+    p.ts_log2 = 0;
+    while ((1u << p.ts_log2) < p.ts) ++p.ts_log2;
+    return p;
+}
+
+struct Layout {
+    size_t F0, F1, S, tile_first, stamp, scan_status, ctl, total;
+};
+
+Layout layout(uint64_t n, uint64_t m, const Params &p) {
+    Layout L;
+    size_t o = 0;
+    auto take = [&](size_t bytes) {
+        size_t at = o;
+        o = align_up(o + bytes);
+        return at;
+    };
+    const uint64_t max_shadows = p.udc ? (m + p.K - 1) / p.K + n : n;   // sum ceil(d/K) <= m/K + |F|
+    const uint64_t max_tiles = (max_shadows + p.ts - 1) / p.ts + 2;
+    const uint64_t max_scan_tiles = (n + kScanTile - 1) / kScanTile + 2;
+    L.F0 = take(4 * (n + 1));
+    L.F1 = take(4 * (n + 1));
+    L.S = take(4 * (n + 2));
+    L.tile_first = take(4 * max_tiles);
+    L.stamp = take(4 * (n + 1));
+    L.scan_status = take(8 * max_scan_tiles);
+    L.ctl = take(sizeof(Ctl));
+    L.total = o;
+    return L;
+}
+
+}  // namespace
+
+struct etg_graph {
+    uint64_t n = 0, m = 0;
+    uint32_t flags = 0;
+    Params p{};
+    const void *off = nullptr;
+    const uint32_t *col = nullptr;
+    const uint32_t *w = nullptr;
+    cudaStream_t stream = nullptr;
+    uint8_t *ws = nullptr;
+    Layout L{};
+    Ctl *ctl = nullptr;
+    int num_sms = 0;
+    int grid_scan = 0;
+    int grid_init = 0;
+    Ctl *h_ctl = nullptr;                 // pinned host mirror for readback
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    cudaGraphExec_t exec[4] = {nullptr, nullptr, nullptr, nullptr};
+    cudaGraph_t graph[4] = {nullptr, nullptr, nullptr, nullptr};
+};
+
+namespace {
+
+template <class OffT>
+Dev<OffT> make_dev(const etg_graph *g) {
+    Dev<OffT> d;
+    d.off = static_cast<const OffT *>(g->off);
+    d.col = g->col;
+    d.w = g->w;
+    d.F[0] = reinterpret_cast<uint32_t *>(g->ws + g->L.F0);
+    d.F[1] = reinterpret_cast<uint32_t *>(g->ws + g->L.F1);
+    d.S = reinterpret_cast<uint32_t *>(g->ws + g->L.S);
+    d.tile_first = reinterpret_cast<uint32_t *>(g->ws + g->L.tile_first);
+    d.stamp = reinterpret_cast<uint32_t *>(g->ws + g->L.stamp);
+    d.scan_status = reinterpret_cast<unsigned long long *>(g->ws + g->L.scan_status);
+    d.ctl = g->ctl;
+    d.n = (uint32_t)g->n;
+    d.K = g->p.K;
+    d.ts = g->p.ts;
+    d.ts_log2 = g->p.ts_log2;
+    return d;
+}
+
+// --- kernel selection ------------------------------------------------------ //
+template <class OffT, int ALG>
+const void *expand_fn(bool udc, bool smp) {
+    if (!udc) return (const void *)expand_kernel<OffT, ALG, false, false>;
+    if (smp) return (const void *)expand_kernel<OffT, ALG, true, true>;
+    return (const void *)expand_kernel<OffT, ALG, true, false>;
+}
+
+template <class OffT>
+const void *expand_fn_alg(int alg, bool udc, bool smp) {
+    switch (alg) {
+        case ALG_BFS: return expand_fn<OffT, ALG_BFS>(udc, smp);
+        case ALG_SSSP: return expand_fn<OffT, ALG_SSSP>(udc, smp);
+        case ALG_CC: return expand_fn<OffT, ALG_CC>(udc, smp);
+        default: return expand_fn<OffT, ALG_SSWP>(udc, smp);
+    }
+}
+
+template <class OffT>
+const void *init_fn(int alg) {
+    switch (alg) {
+        case ALG_BFS: return (const void *)init_kernel<OffT, ALG_BFS>;
+        case ALG_SSSP: return (const void *)init_kernel<OffT, ALG_SSSP>;
+        case ALG_CC: return (const void *)init_kernel<OffT, ALG_CC>;
+        default: return (const void *)init_kernel<OffT, ALG_SSWP>;
+    }
+}
+
+template <class OffT>
+const void *scan_fn(bool udc) {
+    return udc ? (const void *)udc_scan_kernel<OffT, true> : (const void *)udc_scan_kernel<OffT, false>;
+}
+
+size_t expand_smem(const Params &p, int alg) {
+    if (!p.smp) return 0;
+    const size_t cap = (size_t)p.ts * p.K;
+    const bool kw = (alg == ALG_SSSP || alg == ALG_SSWP);
+    return cap * 4 * (kw ? 2 : 1) + cap;
+}
+
+struct Launch {
+    const void *fn;
+    dim3 grid;
+    size_t smem;
+};
+
+template <class OffT>
+etg_status expand_launch(etg_graph *g, int alg, Launch &out) {
+    out.fn = expand_fn_alg<OffT>(alg, g->p.udc, g->p.smp);
+    out.smem = expand_smem(g->p, alg);
+    ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)out.smem));
+    int nb = 0;
+    ETG_CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, out.fn, kBlock, out.smem));
+    if (nb < 1) nb = 1;
+    out.grid = dim3((unsigned)(nb * g->num_sms));
+    return ETG_OK;
+}
+
+// Build the while-loop graph for one algorithm (lazily, cached per handle).
+template <class OffT>
+etg_status build_graph(etg_graph *g, int alg) {
+    if (g->exec[alg]) return ETG_OK;
+    Dev<OffT> d = make_dev<OffT>(g);
+    Launch ex;
+    etg_status s = expand_launch<OffT>(g, alg, ex);
+    if (s != ETG_OK) return s;
+    uint32_t cap_e = g->p.ts * g->p.K;
+    cudaGraph_t graph;
+    ETG_CU(cudaGraphCreate(&graph, 0));
+    cudaGraphConditionalHandle cond;
+    ETG_CU(cudaGraphConditionalHandleCreate(&cond, graph, 1, cudaGraphCondAssignDefault));
+    cudaGraphNodeParams cp = {};
+    cp.type = cudaGraphNodeTypeConditional;
+    cp.conditional.handle = cond;
+    cp.conditional.type = cudaGraphCondTypeWhile;
+    cp.conditional.size = 1;
+    cudaGraphNode_t cnode;
+    ETG_CU(cudaGraphAddNode(&cnode, graph, nullptr, 0, &cp));
+    cudaGraph_t body = cp.conditional.phGraph_out[0];
+
+    cudaKernelNodeParams kp;
+    cudaGraphNode_t n_scan, n_exp, n_adv;
+    void *scan_args[] = {&d};
+    memset(&kp, 0, sizeof(kp));
+    kp.func = const_cast<void *>(scan_fn<OffT>(g->p.udc));
+    kp.gridDim = dim3(g->grid_scan);
+    kp.blockDim = dim3(kBlock);
+    kp.kernelParams = scan_args;
+    ETG_CU(cudaGraphAddKernelNode(&n_scan, body, nullptr, 0, &kp));
+
+    void *exp_args[] = {&d, &cap_e};
+    memset(&kp, 0, sizeof(kp));
+    kp.func = const_cast<void *>(ex.fn);
+    kp.gridDim = ex.grid;
+    kp.blockDim = dim3(kBlock);
+    kp.sharedMemBytes = (unsigned)ex.smem;
+    kp.kernelParams = exp_args;
+    ETG_CU(cudaGraphAddKernelNode(&n_exp, body, &n_scan, 1, &kp));
+
+    Ctl *ctl = g->ctl;
+    int use_cond = 1;
+    void *adv_args[] = {&ctl, &cond, &use_cond};
+    memset(&kp, 0, sizeof(kp));
+    kp.func = (void *)advance_kernel;
+    kp.gridDim = dim3(1);
+    kp.blockDim = dim3(1);
+    kp.kernelParams = adv_args;
+    ETG_CU(cudaGraphAddKernelNode(&n_adv, body, &n_exp, 1, &kp));
+
+    ETG_CU(cudaGraphInstantiate(&g->exec[alg], graph, 0));
+    g->graph[alg] = graph;
+    return ETG_OK;
+}
+
+template <class OffT>
+etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stats *st) {
+    Dev<OffT> d = make_dev<OffT>(g);
+    cudaStream_t s = g->stream;
+    const bool host_loop = (g->flags & ETG_HOST_LOOP) != 0;
+    if (!host_loop) {
+        etg_status rc = build_graph<OffT>(g, alg);
+        if (rc != ETG_OK) return rc;
+    }
+    ETG_CU(cudaEventRecord(g->ev0, s));
+    ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, label, source);
+    {
+        void *args[] = {&d, &label, &source};
+        ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), args, 0, s));
+    }
+    uint64_t launches = 2;
+    if (host_loop) {
+        Launch ex;
+        etg_status rc = expand_launch<OffT>(g, alg, ex);
+        if (rc != ETG_OK) return rc;
+        uint32_t cap_e = g->p.ts * g->p.K;
+        cudaGraphConditionalHandle none = 0;
+        int zero = 0;
+        Ctl *ctl = g->ctl;
+        ETG_CU(cudaMemcpyAsync(&g->h_ctl->count[0], &g->ctl->count[0], 4, cudaMemcpyDeviceToHost, s));
+        ETG_CU(cudaStreamSynchronize(s));
+        uint32_t it = 0;
+        while (g->h_ctl->count[0] > 0) {
+            void *scan_args[] = {&d};
+            ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+            void *exp_args[] = {&d, &cap_e};
+            ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
+            void *adv_args[] = {&ctl, &none, &zero};
+            ETG_CU(cudaLaunchKernel((const void *)advance_kernel, dim3(1), dim3(1), adv_args, 0, s));
+            launches += 3;
+            ++it;
+            // read back the size of the next active set ("actSet.isNotEmpty()", L207)
+            ETG_CU(cudaMemcpyAsync(&g->h_ctl->count[0], &g->ctl->count[it & 1], 4, cudaMemcpyDeviceToHost, s));
+            ETG_CU(cudaStreamSynchronize(s));
+        }
+    } else {
+        ETG_CU(cudaGraphLaunch(g->exec[alg], s));
+    }
+    ETG_CU(cudaEventRecord(g->ev1, s));
+    ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    ETG_CU(cudaStreamSynchronize(s));
+    ETG_CU(cudaGetLastError());
+    if (!host_loop) launches += 3ull * g->h_ctl->iter;
+    g_launches += launches;
+    if (st) {
+        float ms = 0.f;
+        ETG_CU(cudaEventElapsedTime(&ms, g->ev0, g->ev1));
+        st->iterations = g->h_ctl->iterations;
+        st->reserved = 0;
+        st->activations = g->h_ctl->activations;
+        st->shadows = g->h_ctl->shadows;
+        st->edges_processed = g->h_ctl->edges;
+        st->vertices_reached = 0;
+        st->edges_reached = 0;
+        st->ms = ms;
+    }
+    return ETG_OK;
+}
+
+etg_status run(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stats *st) {
+    if (!g || !label) return fail(ETG_EINVAL, "null handle or label pointer");
+    if (alg != ALG_CC && source >= g->n) return fail(ETG_EINVAL, "source >= n");
+    if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "graph loaded without weights");
+    if (alg == ALG_CC && !(g->flags & ETG_SYMMETRIC)) return fail(ETG_ENOTSYM, "etg_cc needs ETG_SYMMETRIC");
+    if (g->n == 0) return ETG_OK;
+    return g->p.u64 ? run_impl<uint64_t>(g, alg, source, label, st)
+                    : run_impl<uint32_t>(g, alg, source, label, st);
+}
+
+template <class OffT>
+etg_status validate_impl(etg_graph *g) {
+    Dev<OffT> d = make_dev<OffT>(g);
+    validate_kernel<OffT><<<g->num_sms * 4, kBlock, 0, g->stream>>>(d, (unsigned long long)g->m);
+    g_launches += 1;
+    ETG_CU(cudaMemcpyAsync(&g->h_ctl->error, &g->ctl->error, 4, cudaMemcpyDeviceToHost, g->stream));
+    ETG_CU(cudaStreamSynchronize(g->stream));
+    if (g->h_ctl->error) return fail(ETG_EINVALID_CSR, "CSR validation failed, code " + std::to_string(g->h_ctl->error));
+    return ETG_OK;
+}
+
+template <class OffT>
+etg_status reach_impl(etg_graph *g, const uint32_t *label, uint32_t unreached, etg_stats *st) {
+    Dev<OffT> d = make_dev<OffT>(g);
+    ETG_CU(cudaMemsetAsync(&g->ctl->reached_v, 0, 16, g->stream));
+    reach_kernel<OffT><<<g->num_sms * 4, kBlock, 0, g->stream>>>(d, label, unreached);
+    g_launches += 1;
+    ETG_CU(cudaMemcpyAsync(&g->h_ctl->reached_v, &g->ctl->reached_v, 16, cudaMemcpyDeviceToHost, g->stream));
+    ETG_CU(cudaStreamSynchronize(g->stream));
+    ETG_CU(cudaGetLastError());
+    st->vertices_reached = g->h_ctl->reached_v;
+    st->edges_reached = g->h_ctl->reached_e;
+    return ETG_OK;
+}
+
+template <class OffT>
+etg_status udc_impl(etg_graph *g, const uint32_t *act, uint32_t n_act, uint32_t *id, uint64_t *start,
+                    uint64_t *end, uint64_t cap, uint64_t *n_out) {
+    Dev<OffT> d = make_dev<OffT>(g);
+    cudaStream_t s = g->stream;
+    ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, nullptr, 0);
+    if (n_act) ETG_CU(cudaMemcpyAsync(d.F[0], act, 4ull * n_act, cudaMemcpyDeviceToDevice, s));
+    ETG_CU(cudaMemcpyAsync(&g->ctl->count[0], &n_act, 4, cudaMemcpyHostToDevice, s));
+    udc_scan_kernel<OffT, true><<<g->grid_scan, kBlock, 0, s>>>(d);
+    ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    ETG_CU(cudaStreamSynchronize(s));
+    *n_out = g->h_ctl->nshadow;
+    if (g->h_ctl->nshadow > cap) return fail(ETG_ENOMEM, "cap too small for the shadow list");
+    udc_dump_kernel<OffT, true><<<g->num_sms * 4, kBlock, 0, s>>>(d, id, start, end);
+    g_launches += 3;
+    ETG_CU(cudaStreamSynchronize(s));
+    ETG_CU(cudaGetLastError());
+    return ETG_OK;
+}
+
+}  // namespace
+
+// =========================================================================== //
+// C ABI
+// =========================================================================== //
+extern "C" {
+
+size_t etg_workspace_bytes(uint64_t n, uint64_t m, const etg_options *opt) {
+    return layout(n, m, derive(opt)).total;
+}
+
+etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_row_offsets,
+                        const uint32_t *d_col_idx, const uint32_t *d_weights, void *d_workspace,
+                        size_t workspace_bytes, void *stream, const etg_options *opt) {
+    if (!out) return fail(ETG_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (!d_row_offsets || (m && !d_col_idx) || !d_workspace) return fail(ETG_EINVAL, "NULL device pointer");
+    const Params p = derive(opt);
+    const uint32_t flags = opt ? opt->flags : 0u;
+    if (n > 0xFFFFFFFEull) return fail(ETG_ERANGE, "n > 2^32 - 2");
+    if (!p.u64 && m > 0xFFFFFFFFull) return fail(ETG_ERANGE, "m >= 2^32 needs ETG_OFFSETS_U64");
+    if (p.udc && p.K == 0) return fail(ETG_EINVAL, "K = 0");
+    const uint64_t max_shadows = p.udc ? (m + p.K - 1) / p.K + n : n;
+    if (max_shadows >= 0xFFFFFFFFull) return fail(ETG_ERANGE, "shadow count may exceed 2^32 (raise K)");
+    const Layout L = layout(n, m, p);
+    if (workspace_bytes < L.total) return fail(ETG_ENOMEM, "workspace too small: need " + std::to_string(L.total));
+    if (reinterpret_cast<uintptr_t>(d_workspace) % kAlign) return fail(ETG_EINVAL, "workspace must be 256-byte aligned");
+
+    etg_graph *g = new (std::nothrow) etg_graph();
+    if (!g) return fail(ETG_ENOMEM, "host allocation failed");
+    g->n = n;
+    g->m = m;
+    g->flags = flags;
+    g->p = p;
+    g->off = d_row_offsets;
+    g->col = d_col_idx;
+    g->w = d_weights;
+    g->stream = static_cast<cudaStream_t>(stream);
+    g->ws = static_cast<uint8_t *>(d_workspace);
+    g->L = L;
+    g->ctl = reinterpret_cast<Ctl *>(g->ws + L.ctl);
+    auto bail = [&](etg_status s) {
+        etg_free(g);
+        return s;
+    };
+    int dev = 0;
+    cudaError_t e;
+    if ((e = cudaGetDevice(&dev)) != cudaSuccess ||
+        (e = cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess ||
+        (e = cudaMallocHost(&g->h_ctl, sizeof(Ctl))) != cudaSuccess ||
+        (e = cudaEventCreate(&g->ev0)) != cudaSuccess || (e = cudaEventCreate(&g->ev1)) != cudaSuccess ||
+        (e = cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), g->stream)) != cudaSuccess ||
+        (e = cudaMemsetAsync(g->ws + L.stamp, 0, 4 * (n + 1), g->stream)) != cudaSuccess ||
+        (e = cudaMemsetAsync(g->ws + L.scan_status, 0, L.ctl - L.scan_status, g->stream)) != cudaSuccess) {
+        return bail(fail(ETG_ECUDA, std::string("load: ") + cudaGetErrorString(e)));
+    }
+    g->grid_scan = g->num_sms * 2;
+    g->grid_init = g->num_sms * 8;
+    if (flags & ETG_VALIDATE) {
+        etg_status s = p.u64 ? validate_impl<uint64_t>(g) : validate_impl<uint32_t>(g);
+        if (s != ETG_OK) return bail(s);
+    }
+    if ((e = cudaStreamSynchronize(g->stream)) != cudaSuccess)
+        return bail(fail(ETG_ECUDA, std::string("load sync: ") + cudaGetErrorString(e)));
+    *out = g;
+    return ETG_OK;
+}
+
+etg_status etg_bfs(etg_graph *g, uint32_t source, uint32_t *d_depth, etg_stats *st) {
+    return run(g, ALG_BFS, source, d_depth, st);
+}
+
+etg_status etg_sssp(etg_graph *g, uint32_t source, uint32_t *d_dist, etg_stats *st) {
+    return run(g, ALG_SSSP, source, d_dist, st);
+}
+
+etg_status etg_cc(etg_graph *g, uint32_t *d_label, etg_stats *st) {
+    return run(g, ALG_CC, 0, d_label, st);
+}
+
+etg_status etg_sswp(etg_graph *g, uint32_t source, uint32_t *d_width, etg_stats *st) {
+    return run(g, ALG_SSWP, source, d_width, st);
+}
+
+etg_status etg_reach_stats(etg_graph *g, const uint32_t *d_label, uint32_t unreached, etg_stats *st) {
+    if (!g || !d_label || !st) return fail(ETG_EINVAL, "NULL argument");
+    if (g->n == 0) {
+        st->vertices_reached = st->edges_reached = 0;
+        return ETG_OK;
+    }
+    return g->p.u64 ? reach_impl<uint64_t>(g, d_label, unreached, st)
+                    : reach_impl<uint32_t>(g, d_label, unreached, st);
+}
+
+etg_status etg_udc_slices(etg_graph *g, const uint32_t *d_active, uint32_t n_active, uint32_t *d_id,
+                          uint64_t *d_start, uint64_t *d_end, uint64_t cap, uint64_t *n_out) {
+    if (!g || !n_out || (n_active && !d_active)) return fail(ETG_EINVAL, "NULL argument");
+    if (!g->p.udc) return fail(ETG_EINVAL, "etg_udc_slices needs a UDC handle");
+    if (n_active > g->n) return fail(ETG_EINVAL, "active set larger than n");
+    return g->p.u64 ? udc_impl<uint64_t>(g, d_active, n_active, d_id, d_start, d_end, cap, n_out)
+                    : udc_impl<uint32_t>(g, d_active, n_active, d_id, d_start, d_end, cap, n_out);
+}
+
+void etg_free(etg_graph *g) {
+    if (!g) return;
+    for (int a = 0; a < 4; ++a) {
+        if (g->exec[a]) cudaGraphExecDestroy(g->exec[a]);
+        if (g->graph[a]) cudaGraphDestroy(g->graph[a]);
+    }
+    if (g->ev0) cudaEventDestroy(g->ev0);
+    if (g->ev1) cudaEventDestroy(g->ev1);
+    if (g->h_ctl) cudaFreeHost(g->h_ctl);
+    delete g;
+}
+
+size_t etg_host_scratch_bytes(uint64_t n, uint64_t m, int has_weights, const etg_options *opt) {
+    const Params p = derive(opt);
+    size_t o = 0;
+    o = align_up(o + (p.u64 ? 8 : 4) * (n + 1));
+    o = align_up(o + 4 * m);
+    if (has_weights) o = align_up(o + 4 * m);
+    o = align_up(o + 4 * n);
+    return o + layout(n, m, p).total;
+}
+
+etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_off, const uint32_t *h_col,
+                        const uint32_t *h_w, uint32_t source, uint32_t *h_labels, void *d_scratch,
+                        size_t scratch_bytes, void *stream, const etg_options *opt, etg_stats *st) {
+    if (!h_off || (m && !h_col) || !h_labels || !d_scratch) return fail(ETG_EINVAL, "NULL argument");
+    if (alg < 0 || alg > 3) return fail(ETG_EINVAL, "alg must be 0..3");
+    const Params p = derive(opt);
+    const bool has_w = (alg == ALG_SSSP || alg == ALG_SSWP);
+    if (has_w && !h_w) return fail(ETG_ENOWEIGHTS, "weights required");
+    if (scratch_bytes < etg_host_scratch_bytes(n, m, has_w, opt)) return fail(ETG_ENOMEM, "scratch too small");
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    uint8_t *base = static_cast<uint8_t *>(d_scratch);
+    size_t o = 0;
+    const size_t offsz = (p.u64 ? 8 : 4) * (n + 1);
+    uint8_t *d_off = base + o;
+    o = align_up(o + offsz);
+    uint32_t *d_col = reinterpret_cast<uint32_t *>(base + o);
+    o = align_up(o + 4 * m);
+    uint32_t *d_w = nullptr;
+    if (has_w) {
+        d_w = reinterpret_cast<uint32_t *>(base + o);
+        o = align_up(o + 4 * m);
+    }
+    uint32_t *d_lab = reinterpret_cast<uint32_t *>(base + o);
+    o = align_up(o + 4 * n);
+    ETG_CU(cudaMemcpyAsync(d_off, h_off, offsz, cudaMemcpyHostToDevice, s));
+    if (m) ETG_CU(cudaMemcpyAsync(d_col, h_col, 4 * m, cudaMemcpyHostToDevice, s));
+    if (has_w && m) ETG_CU(cudaMemcpyAsync(d_w, h_w, 4 * m, cudaMemcpyHostToDevice, s));
+    etg_graph *g = nullptr;
+    etg_status rc = etg_load_csr(&g, n, m, d_off, d_col, d_w, base + o, scratch_bytes - o, stream, opt);
+    if (rc != ETG_OK) return rc;
+    rc = run(g, alg, source, d_lab, st);
+    if (rc == ETG_OK) {
+        cudaError_t e = cudaMemcpyAsync(h_labels, d_lab, 4 * n, cudaMemcpyDeviceToHost, s);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+        if (e != cudaSuccess) rc = fail(ETG_ECUDA, std::string("run_host D2H: ") + cudaGetErrorString(e));
+    }
+    etg_free(g);
+    return rc;
+}
+
+const char *etg_status_str(etg_status s) {
+    switch (s) {
+        case ETG_OK: return "ETG_OK";
+        case ETG_EINVAL: return "ETG_EINVAL";
+        case ETG_ENOMEM: return "ETG_ENOMEM";
+        case ETG_ECUDA: return "ETG_ECUDA";
+        case ETG_ENCCL: return "ETG_ENCCL";
+        case ETG_ENOTSYM: return "ETG_ENOTSYM";
+        case ETG_ERANGE: return "ETG_ERANGE";
+        case ETG_ENOWEIGHTS: return "ETG_ENOWEIGHTS";
+        case ETG_EINVALID_CSR: return "ETG_EINVALID_CSR";
+    }
+    return "unknown";
+}
+
+const char *etg_last_error(void) { return g_err.c_str(); }
+
+uint64_t etg_kernel_launches(void) { return g_launches.load(); }
+
+}  // extern "C"

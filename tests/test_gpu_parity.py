@@ -1,0 +1,265 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle, bit-exact.
+
+All labels are integers, and every result is a unique fixpoint (SURVEY 8(c)
+"GPU = oracle"), so the bar is element-by-element equality of the n labels.
+"""
+import numpy as np
+import pytest
+import torch
+
+import graphgen as gg
+import oracle
+from etg_testutil import load_golden, to_etg
+
+pytestmark = pytest.mark.gpu
+
+etg = pytest.importorskip("paper_conf_ipps_wangzlg19_b200")
+U32 = etg.to_u32_numpy
+INF = etg.INF
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _built():
+    from paper_conf_ipps_wangzlg19_b200 import _build
+    _build.build()
+    assert torch.cuda.is_available()
+
+
+def check_all(g, sources, K=32, flags=0, algs=("bfs", "sssp", "sswp"), force_u64=False):
+    off, col, w = g.numpy()
+    G = to_etg(g, K=K, flags=flags, force_u64=force_u64)
+    for s in sources:
+        if "bfs" in algs:
+            got, st = G.bfs(s)
+            exp = oracle.bfs(off, col, s)
+            np.testing.assert_array_equal(U32(got), exp, err_msg=f"BFS s={s} K={K} flags={flags}")
+        if "sssp" in algs and w is not None:
+            got, st = G.sssp(s)
+            np.testing.assert_array_equal(U32(got), oracle.sssp(off, col, w, s),
+                                          err_msg=f"SSSP s={s} K={K} flags={flags}")
+        if "sswp" in algs and w is not None:
+            got, st = G.sswp(s)
+            np.testing.assert_array_equal(U32(got), oracle.sswp(off, col, w, s),
+                                          err_msg=f"SSWP s={s} K={K} flags={flags}")
+    return G
+
+
+def check_cc(gs, K=32, flags=0):
+    soff, scol, _ = gs.numpy()
+    G = to_etg(gs, K=K, flags=flags, symmetric=True)
+    got, st = G.cc()
+    np.testing.assert_array_equal(U32(got), oracle.cc(soff, scol), err_msg=f"CC K={K} flags={flags}")
+    return st
+
+
+# --------------------------------------------------------------------------- #
+# golden fixtures
+# --------------------------------------------------------------------------- #
+def _fixture_graph(f, key_w="w"):
+    off = torch.tensor(f["off"], dtype=torch.int64)
+    col = torch.tensor(f["col"], dtype=torch.int64)
+    w = torch.tensor(f[key_w], dtype=torch.int64) if key_w in f else None
+    return gg.Graph(f["id"], f["n"], off, col, w)
+
+
+def test_golden_f1_bfs_udc_cc():
+    f = load_golden("F1_fig3_udc.json")
+    g = _fixture_graph(f)
+    G = to_etg(g, K=f["K"])
+    got, _ = G.bfs(f["bfs_source"])
+    assert U32(got).tolist() == f["expect_bfs"]
+    ids, st, en = G.udc_slices(torch.tensor(f["active"][:1] + f["active"][2:], device="cuda"))
+    got = [[int(a), int(b), int(c)] for a, b, c in zip(U32(ids), st.cpu(), en.cpu())]
+    assert got == f["expect_shadows"]                      # vertex 2 (degree 0) is filtered (L142)
+    gs = gg.symmetrize(g)
+    check_cc(gs, K=f["K"])
+
+
+def test_golden_f2_f4():
+    f = load_golden("F2_sssp_reactivation.json")
+    G = to_etg(_fixture_graph(f))
+    assert U32(G.bfs(f["source"])[0]).tolist() == f["expect_bfs"]
+    assert U32(G.sssp(f["source"])[0]).tolist() == f["expect_sssp"]
+    f = load_golden("F4_saturation.json")
+    G = to_etg(_fixture_graph(f))
+    assert U32(G.sssp(f["source"])[0]).tolist() == f["expect_sssp"]
+
+
+def test_golden_f3_cc():
+    f = load_golden("F3_cc_weak.json")
+    g = gg.from_edges("F3", f["n"], f["edges"])
+    gs = gg.symmetrize(g)
+    G = to_etg(gs, symmetric=True)
+    assert U32(G.cc()[0]).tolist() == f["expect_cc"]
+
+
+# --------------------------------------------------------------------------- #
+# C1 (the parity config) and the K / UDC / SMP / control sweeps
+# --------------------------------------------------------------------------- #
+@pytest.fixture(scope="module")
+def c1():
+    return gg.make("C1")
+
+
+@pytest.fixture(scope="module")
+def c1sym():
+    return gg.make("C1", symmetric=True, weights=False)
+
+
+def test_c1_all_algorithms(c1, c1sym):
+    srcs = [gg.first_source(c1)] + gg.sample_sources(c1, 4, 11)
+    check_all(c1, srcs)
+    check_cc(c1sym)
+
+
+@pytest.mark.parametrize("K", [1, 2, 3, 4, 10, 31, 32, 33, 64, 128, 1024])
+def test_k_invariance(c1, c1sym, K):
+    """Theorems 1-2 (L119-127): labels identical for every degree limit K."""
+    srcs = gg.sample_sources(c1, 2, K)
+    check_all(c1, srcs, K=K)
+    check_cc(c1sym, K=K)
+
+
+@pytest.mark.parametrize("flags", [2, 4, 32, 2 | 32, 4 | 32])
+def test_flag_invariance(c1, c1sym, flags):
+    """UDC off (L88 baseline), SMP off (Fig. 6 ablation), host-driven loop."""
+    srcs = gg.sample_sources(c1, 2, 5)
+    check_all(c1, srcs, flags=flags)
+    check_cc(c1sym, flags=flags)
+
+
+def test_u64_offsets(c1):
+    check_all(c1, gg.sample_sources(c1, 2, 3), force_u64=True)
+
+
+@pytest.mark.parametrize("cfg", ["T14", "LJ-small"])
+def test_other_shapes(cfg):
+    g = gg.make(cfg)
+    check_all(g, gg.sample_sources(g, 3, 2))
+    check_cc(gg.make(cfg, symmetric=True, weights=False))
+
+
+# --------------------------------------------------------------------------- #
+# edge cases
+# --------------------------------------------------------------------------- #
+def test_source_with_zero_outdegree(c1):
+    deg = c1.degrees()
+    s = int(torch.nonzero(deg == 0)[0, 0])
+    G = to_etg(c1)
+    got = U32(G.bfs(s)[0])
+    assert got[s] == 0 and np.sum(got != INF) == 1
+    assert U32(G.sswp(s)[0])[s] == INF
+
+
+def test_tiny_and_empty_graphs():
+    g = gg.from_edges("one", 1, [])
+    G = to_etg(g)
+    assert U32(G.bfs(0)[0]).tolist() == [0]
+    g = gg.from_edges("two", 2, [(0, 1)], weights=[7])
+    G = to_etg(g)
+    assert U32(G.sssp(0)[0]).tolist() == [0, 7]
+    assert U32(G.sssp(1)[0]).tolist() == [INF, 0]
+
+
+def test_hub_spanning_many_tiles():
+    """One hub with 300K out-edges: UDC cuts it into ~9.4K shadows over ~37 tiles."""
+    n = 400_000
+    hub = [(0, v) for v in range(1, 300_001)]
+    tail = [(v, v + 1) for v in range(300_000, n - 1)]
+    g = gg.add_weights(gg.from_edges("hub", n, hub + tail), 99)
+    check_all(g, [0, 5, 300_000], algs=("bfs", "sssp"))
+    check_all(g, [0], K=1, algs=("bfs",))
+
+
+def test_in_degree_skew():
+    """All edges into one vertex: heavy atomic contention on a single label."""
+    n = 50_000
+    e = [(v, 0) for v in range(1, n)] + [(0, v) for v in range(1, n, 7)]
+    g = gg.add_weights(gg.from_edges("sink", n, e), 5)
+    check_all(g, [1, 0], algs=("bfs", "sssp"))
+    check_cc(gg.symmetrize(gg.from_edges("sink", n, e)))
+
+
+def test_duplicates_and_self_loops_tolerated():
+    e = [(0, 1), (0, 1), (1, 1), (1, 2), (2, 0), (2, 3), (2, 3)]
+    g = gg.add_weights(gg.from_edges("dup", 5, e), 1)
+    check_all(g, [0, 2])
+
+
+def test_large_weights_saturate():
+    n = 64
+    e = [(i, i + 1) for i in range(n - 1)]
+    g = gg.from_edges("sat", n, e, weights=[2**31 - 1] * (n - 1))
+    check_all(g, [0], algs=("sssp",))
+
+
+# --------------------------------------------------------------------------- #
+# step A2 (UDC) through the library's own device mapping
+# --------------------------------------------------------------------------- #
+@pytest.mark.parametrize("K", [1, 4, 10, 32, 33, 1000])
+def test_udc_slices_match_oracle(K):
+    g = gg.make("LJ-small", weights=False)
+    off, _, _ = g.numpy()
+    deg = np.diff(off.astype(np.int64))
+    cand = np.nonzero(deg > 0)[0]
+    rng = np.random.default_rng(K)
+    act = rng.choice(cand, size=5000, replace=False).astype(np.int64)
+    act = np.concatenate([act, [int(np.argmax(deg))]])
+    G = to_etg(g, K=K)
+    ids, st, en = G.udc_slices(torch.from_numpy(act).cuda())
+    eid, est, een = oracle.udc_slices(off, act.astype(np.uint32), K)
+    np.testing.assert_array_equal(U32(ids), eid)
+    np.testing.assert_array_equal(st.cpu().numpy().astype(np.uint64), est)
+    np.testing.assert_array_equal(en.cpu().numpy().astype(np.uint64), een)
+
+
+# --------------------------------------------------------------------------- #
+# statistics and the host-buffer entry
+# --------------------------------------------------------------------------- #
+def test_bfs_work_counters(c1):
+    """L152: for BFS every reached vertex is active once; edges processed =
+    m of the activatable subgraph; shadows = sum ceil(deg/K) over reached."""
+    off, col, _ = c1.numpy()
+    s = gg.first_source(c1)
+    K = 16
+    G = to_etg(c1, K=K)
+    lab, st = G.bfs(s)
+    exp = oracle.bfs(off, col, s)
+    deg = np.diff(off.astype(np.int64))
+    reached = exp != INF
+    rs = G.reach_stats(lab)
+    assert rs.vertices_reached == int(reached.sum())
+    assert rs.edges_reached == int(deg[reached].sum())
+    assert st.edges_processed == int(deg[reached].sum())
+    assert st.shadows == int(((deg[reached] + K - 1) // K).sum())
+    assert st.activations == int(reached.sum()) - 1
+    # the level-d active set is non-empty iff some depth-d vertex has out-edges
+    assert st.iterations == int(exp[reached & (deg > 0)].max()) + 1
+
+
+def test_run_host_matches(c1):
+    off, col, w = c1.numpy()
+    s = gg.first_source(c1)
+    o = torch.from_numpy(off.astype(np.int64)).to(torch.int32).pin_memory()
+    c = torch.from_numpy(col.view(np.int32)).pin_memory()
+    ww = torch.from_numpy(w.view(np.int32)).pin_memory()
+    out = torch.empty(c1.n, dtype=torch.int32).pin_memory()
+    scratch = torch.empty(etg.host_scratch_bytes(c1.n, c1.m, True), dtype=torch.uint8, device="cuda")
+    etg.run_host(etg.SSSP, o, c, ww, s, out, scratch)
+    np.testing.assert_array_equal(out.numpy().view(np.uint32), oracle.sssp(off, col, w, s))
+    etg.run_host(etg.BFS, o, c, None, s, out, scratch)
+    np.testing.assert_array_equal(out.numpy().view(np.uint32), oracle.bfs(off, col, s))
+
+
+def test_errors():
+    g = gg.from_edges("x", 3, [(0, 1)])
+    G = to_etg(g)
+    with pytest.raises(etg.EtgError, match="EINVAL"):
+        G.bfs(5)
+    with pytest.raises(etg.EtgError, match="ENOWEIGHTS"):
+        G.sssp(0)
+    with pytest.raises(etg.EtgError, match="ENOTSYM"):
+        G.cc()
+    bad = gg.Graph("bad", 3, torch.tensor([0, 1, 1, 1]), torch.tensor([7]))
+    with pytest.raises(etg.EtgError, match="EINVALID_CSR"):
+        to_etg(bad)
