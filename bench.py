@@ -1,0 +1,514 @@
+#!/usr/bin/env python
+"""bench.py -- GTEPS of the EtaGraph hot path (BFS + SSSP + CC) on B200.
+
+One STEP = one pass of the whole hot path (rows A1-A7 of SURVEY 8(a)) for each
+algorithm on the N=1 workload, BASELINE.json configs[1] = C2 (RMAT scale 22,
+edge factor 16, PaRMAT a/b/c = .45/.22/.22): one BFS and one SSSP from the same
+seeded source (16 sources, rotating) and one CC on the symmetrised graph.
+
+value = traversed edges / device time, summed over the step's three calls
+(GTEPS; edges = m of the activatable subgraph for BFS/SSSP, Def. 2, and
+nnz of the symmetric CSR for CC).  Inputs are resident in HBM; L2 is flushed
+(256 MiB write) before every traversal call, outside the timed events.
+
+Under torchrun (N > 1) every rank runs its own sources on its own GPU
+(independent problems, no data-path collective): "scaling": "weak", value =
+edges of all ranks / max over ranks of the device time.
+
+--impl reference times the CPU oracle (oracle/, the paper's definitions written
+out plainly) on the host cores, on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import ctypes
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "GTEPS (BFS/SSSP/CC) at 1/2/4/8 B200; expand-kernel HBM GB/s vs peak"
+UNIT = "GTEPS"
+# algorithmic bytes: per relaxed edge, per active vertex
+BYTES_PER_EDGE = {"bfs": 8, "sssp": 12, "cc": 8}
+BYTES_PER_VERTEX = {"bfs": 20, "sssp": 24, "cc": 24}
+REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+           0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+           0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+           0x100: "display_clock_setting"}
+
+
+def parse_args():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    p.add_argument("--config", default="C2")
+    p.add_argument("--algs", default="bfs,sssp,cc")
+    p.add_argument("--K", type=int, default=32)
+    p.add_argument("--flags", type=int, default=0, help="extra ETG_* flags (e.g. 2 = NO_UDC)")
+    p.add_argument("--sources", type=int, default=16)
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-profile", action="store_true")
+    p.add_argument("--json-out", default=None)
+    return p.parse_args()
+
+
+# --------------------------------------------------------------------------- #
+# distributed plumbing
+# --------------------------------------------------------------------------- #
+def dist_setup():
+    import torch
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    elif torch.cuda.is_available():
+        torch.cuda.set_device(0)
+    return rank, world, local
+
+
+def barrier(world):
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def allreduce(vals, op, world):
+    if world == 1:
+        return vals
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor(vals, dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=op)
+    return t.tolist()
+
+
+# --------------------------------------------------------------------------- #
+# clocks during the timed region
+# --------------------------------------------------------------------------- #
+class ClockSampler:
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.path = None
+        self.t0 = self.t1 = None
+
+    def start(self):
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index),
+                 "--query-gpu=timestamp,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active",
+                 "--format=csv,noheader,nounits", "-lms", "50"],
+                stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except OSError:
+            self.proc = None
+
+    def mark(self, which):
+        setattr(self, which, time.time())
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        time.sleep(0.12)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        rows = []
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 5:
+                continue
+            try:
+                ts = time.mktime(time.strptime(parts[0].split(".")[0], "%Y/%m/%d %H:%M:%S"))
+                ts += float("0." + parts[0].split(".")[1]) if "." in parts[0] else 0.0
+                rows.append((ts, float(parts[1]), float(parts[2]), float(parts[3]), int(parts[4], 16)))
+            except (ValueError, IndexError):
+                continue
+        os.unlink(self.path)
+        if not rows:
+            return None
+        inside = [r for r in rows if self.t0 - 0.06 <= r[0] <= self.t1 + 0.06] or rows
+        busy = [r for r in inside if not (r[4] & 0x1)] or inside
+        reasons = set()
+        for r in inside:
+            for bit, name in REASONS.items():
+                if r[4] & bit and bit != 0x1:
+                    reasons.add(name)
+        return {"sm_mhz": statistics.median(r[1] for r in busy), "sm_max_mhz": max(r[2] for r in inside),
+                "reasons": sorted(reasons), "samples": len(inside),
+                "power_w_max": max(r[3] for r in inside)}
+
+
+def measured_peak():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    except (OSError, KeyError, ValueError):
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(config):
+    """dram bytes per expand launch from the committed ncu --set full summary, if any."""
+    path = os.path.join(ROOT, "profiles", "expand_ncu_summary.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return d.get(config, {}).get("dram_bytes_per_launch")
+    except (OSError, ValueError):
+        return None
+
+
+# --------------------------------------------------------------------------- #
+# workload
+# --------------------------------------------------------------------------- #
+def build_workload(cfg, device, algs):
+    import graphgen as gg
+    g = gg.make(cfg, device=device, weights=("sssp" in algs))
+    gs = gg.make(cfg, device=device, symmetric=True, weights=False) if "cc" in algs else None
+    return g, gs
+
+
+def oracle_leg(cfg, algs, nsrc, seed, budget_s=25.0, g=None, gs=None):
+    """Time the CPU oracle on a bounded sample: the algorithms of one step, from
+    as many sources as fit in ``budget_s`` (at least one).  Returns (edges, seconds, sample)."""
+    import numpy as np
+    import graphgen as gg
+    import oracle
+    if g is None:
+        g, gs = build_workload(cfg, "cuda" if _has_cuda() else "cpu", algs)
+    off, col, w = g.to("cpu").numpy()
+    deg = np.diff(off.astype(np.int64))
+    srcs = gg.sample_sources(g, nsrc, seed)
+    edges = 0
+    secs = 0.0
+    done = []
+    if gs is not None:
+        soff, scol, _ = gs.to("cpu").numpy()
+    k = 0
+    while True:
+        s = srcs[k % len(srcs)]
+        for a in algs:
+            t = time.perf_counter()
+            if a == "bfs":
+                lab = oracle.bfs(off, col, s)
+            elif a == "sssp":
+                lab = oracle.sssp(off, col, w, s)
+            else:
+                lab = oracle.cc(soff, scol)
+            secs += time.perf_counter() - t
+            if a == "cc":
+                edges += int(scol.shape[0])
+            else:
+                edges += int(deg[lab != oracle.INF].sum())
+            done.append(a if a == "cc" else f"{a}(s={s})")
+        k += 1
+        if secs >= budget_s or k >= len(srcs):
+            break
+    return edges, secs, ", ".join(done)
+
+
+def _has_cuda():
+    try:
+        import torch
+        return torch.cuda.is_available()
+    except ImportError:
+        return False
+
+
+def config_desc(cfg):
+    import graphgen as gg
+    p = gg.CONFIGS[cfg]
+    if p["kind"] == "rmat":
+        return f"{cfg}: RMAT scale-{p['scale']} ef{p['edge_factor']} (PaRMAT a/b/c=.45/.22/.22), seed {p['seed']}"
+    return f"{cfg}: Chung-Lu n={p['n']} m~{p['m_target']} (alpha_out {p['alpha_out']}, alpha_in {p['alpha_in']})"
+
+
+# --------------------------------------------------------------------------- #
+# arms
+# --------------------------------------------------------------------------- #
+def run_reference(args):
+    """The oracle as the reference arm: step i runs ONE call of the step's
+    algorithm set (algs[i % len(algs)], rotating sources), so a default run
+    stays within a few minutes on one host core."""
+    import numpy as np
+    import graphgen as gg
+    import oracle
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    algs = args.algs.split(",")
+    g, gs = build_workload(args.config, "cuda" if _has_cuda() else "cpu", algs)
+    off, col, w = g.to("cpu").numpy()
+    deg = np.diff(off.astype(np.int64))
+    if gs is not None:
+        soff, scol, _ = gs.to("cpu").numpy()
+    srcs = gg.sample_sources(g, args.sources, 4242)
+    edges, secs, done = 0, 0.0, []
+    for i in range(args.warmup + args.steps):
+        a = algs[i % len(algs)]
+        s = srcs[(i // len(algs)) % len(srcs)]
+        if i < args.warmup and i > 0:
+            continue                       # nothing to warm on the CPU beyond one call
+        t = time.perf_counter()
+        if a == "bfs":
+            lab = oracle.bfs(off, col, s)
+        elif a == "sssp":
+            lab = oracle.sssp(off, col, w, s)
+        else:
+            lab = oracle.cc(soff, scol)
+        dt = time.perf_counter() - t
+        if i < args.warmup:
+            continue
+        secs += dt
+        edges += int(scol.shape[0]) if a == "cc" else int(deg[lab != oracle.INF].sum())
+        done.append(a)
+    value = edges / secs / 1e9
+    counts = {a: done.count(a) for a in algs}
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs * 1e3 / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+        "data": "synthetic",
+        "config": {"workload": config_desc(args.config) + "; " + "+".join(algs) + " per step",
+                   "n": g.n, "m": g.m},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                         "sample": f"one oracle call per step, rotating {'/'.join(algs)} and sources: "
+                                   f"{counts} calls on {args.config}"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_ours(args):
+    import numpy as np
+    import torch
+    import torch.distributed as tdist
+    import graphgen as gg
+    import paper_conf_ipps_wangzlg19_b200 as etg
+    from paper_conf_ipps_wangzlg19_b200 import _build
+
+    if not torch.cuda.is_available():
+        print(json.dumps({"metric": METRIC, "error": "no CUDA device (etg has no CPU fallback)"}))
+        return 1
+    rank, world, local = dist_setup()
+    if rank == 0:
+        _build.build()
+    barrier(world)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    algs = args.algs.split(",")
+    g, gs = build_workload(args.config, dev, algs)
+    sources = gg.sample_sources(g, args.sources, 4242 + 7919 * rank)
+
+    def mk(graph, flags, sym=False):
+        o, c, w, fl = etg.csr_to_device(graph.off, graph.col, graph.w, device=dev)
+        return etg.Graph(o, c, w, n=graph.n, K=args.K, flags=flags | fl | args.flags, symmetric=sym)
+
+    G = mk(g, 0)
+    Gs = mk(gs, 0, sym=True) if gs is not None else None
+    out = torch.empty(g.n, dtype=torch.int32, device=dev)
+    # m of the activatable subgraph per source (outside the timed region)
+    m_reach = {}
+    for s in sources:
+        lab, _ = G.bfs(s, out)
+        m_reach[s] = int(G.reach_stats(lab).edges_reached)
+    m_sym = gs.m if gs is not None else 0
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def call(alg, s, handle_main, handle_sym):
+        if alg == "bfs":
+            return handle_main.bfs(s, out)[1], m_reach[s]
+        if alg == "sssp":
+            return handle_main.sssp(s, out)[1], m_reach[s]
+        return handle_sym.cc(out)[1], m_sym
+
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in algs]
+
+    def step(i, acc):
+        s = sources[i % len(sources)]
+        for k, a in enumerate(algs):
+            flush.zero_()
+            evs[k][0].record(stream)
+            st, edges = call(a, s, G, Gs)
+            evs[k][1].record(stream)
+            torch.cuda.synchronize()
+            if acc is not None:
+                ms = evs[k][0].elapsed_time(evs[k][1])
+                acc[a]["ms"] += ms
+                acc[a]["edges"] += edges
+                acc[a]["calls"] += 1
+
+    for i in range(args.warmup):
+        step(i, None)
+    clocks = ClockSampler(torch.cuda.current_device()) if rank == 0 else None
+    if clocks:
+        clocks.start()
+        time.sleep(0.3)
+    acc = {a: {"ms": 0.0, "edges": 0, "calls": 0} for a in algs}
+    launches0 = etg.kernel_launches()
+    barrier(world)
+    torch.cuda.synchronize()
+    if clocks:
+        clocks.mark("t0")
+    for i in range(args.steps):
+        step(args.warmup + i, acc)
+    torch.cuda.synchronize()
+    barrier(world)
+    if clocks:
+        clocks.mark("t1")
+    launches = etg.kernel_launches() - launches0
+    clk = clocks.stop() if clocks else None
+
+    my_ms = sum(v["ms"] for v in acc.values())
+    my_edges = sum(v["edges"] for v in acc.values())
+    max_ms = allreduce([my_ms], tdist.ReduceOp.MAX if world > 1 else None, world)[0]
+    tot_edges = allreduce([float(my_edges)], tdist.ReduceOp.SUM if world > 1 else None, world)[0]
+    per_alg = {}
+    for a in algs:
+        ms_a = allreduce([acc[a]["ms"]], tdist.ReduceOp.MAX if world > 1 else None, world)[0]
+        e_a = allreduce([float(acc[a]["edges"])], tdist.ReduceOp.SUM if world > 1 else None, world)[0]
+        per_alg[a] = {"gteps": e_a / ms_a / 1e6, "ms_per_call": acc[a]["ms"] / max(1, acc[a]["calls"])}
+    value = tot_edges / max_ms / 1e6
+
+    # ---- roofline pass: CUDA events around every expand launch (ETG_PROFILE) ----
+    roof = None
+    if not args.no_profile:
+        Gp = mk(g, etg.PROFILE)
+        Gsp = mk(gs, etg.PROFILE, sym=True) if gs is not None else None
+        bytes_tot, exp_ms, scan_ms, call_ms, launches_p = 0, 0.0, 0.0, 0.0, 0
+        per = {}
+        for i in range(args.steps):
+            s = sources[(args.warmup + i) % len(sources)]
+            for a in algs:
+                flush.zero_()
+                torch.cuda.synchronize()
+                st, _ = call(a, s, Gp, Gsp)
+                b = BYTES_PER_EDGE[a] * st.edges_processed + BYTES_PER_VERTEX[a] * st.frontier_total
+                bytes_tot += b
+                exp_ms += st.expand_ms
+                scan_ms += st.scan_ms
+                call_ms += st.ms
+                launches_p += st.expand_launches
+                d = per.setdefault(a, {"bytes": 0, "expand_ms": 0.0, "launches": 0, "edges_processed": 0})
+                d["bytes"] += b
+                d["expand_ms"] += st.expand_ms
+                d["launches"] += st.expand_launches
+                d["edges_processed"] += st.edges_processed
+        peak, peak_src = measured_peak()
+        achieved = bytes_tot / (exp_ms * 1e-3) / 1e9
+        traffic = ncu_traffic(args.config)
+        roof = {"bound": "hbm", "kernel": "expand_kernel", "achieved": achieved, "peak": peak,
+                "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                "peak_source": peak_src,
+                "algorithmic_bytes_per_launch": bytes_tot / max(1, launches_p),
+                "avg_launch_ms": exp_ms / max(1, launches_p),
+                "expand_share_of_call": exp_ms / max(1e-9, call_ms),
+                "scan_share_of_call": scan_ms / max(1e-9, call_ms),
+                "bytes_model": "BFS 8 B/edge + 20 B/active vertex; SSSP 12 + 24; CC 8 + 24 (SURVEY 8(d))",
+                "timing": "CUDA events on the handle stream around each expand launch (ETG_PROFILE "
+                          "host-driven pass over the same steps)",
+                "per_alg": {a: {"achieved_gbs": v["bytes"] / (v["expand_ms"] * 1e-3) / 1e9,
+                                "launches": v["launches"],
+                                "edges_processed": v["edges_processed"]} for a, v in per.items()}}
+        Gp.close()
+        if Gsp:
+            Gsp.close()
+
+    # ---- e2e: the same metric through the C ABI on HOST buffers ----
+    e2e = None
+    if not args.no_e2e:
+        def pinned(graph):
+            o, c, w, fl = etg.csr_to_device(graph.off, graph.col, graph.w, device="cpu")
+            return (o.pin_memory(), c.pin_memory(), None if w is None else w.pin_memory())
+        hg = pinned(g)
+        hgs = pinned(gs) if gs is not None else None
+        hout = torch.empty(g.n, dtype=torch.int32).pin_memory()
+        scratch = torch.empty(etg.host_scratch_bytes(g.n, max(g.m, m_sym), True, args.K),
+                              dtype=torch.uint8, device=dev)
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e_ms, e_edges, h2d, d2h = 0.0, 0, 0, 0
+        alg_id = {"bfs": etg.BFS, "sssp": etg.SSSP, "cc": etg.CC}
+        for i in range(args.steps):
+            s = sources[(args.warmup + i) % len(sources)]
+            for a in algs:
+                o, c, w = hgs if a == "cc" else hg
+                ww = w if a == "sssp" else None
+                flush.zero_()
+                torch.cuda.synchronize()
+                ev0.record(stream)
+                etg.run_host(alg_id[a], o, c, ww, 0 if a == "cc" else s, hout, scratch, K=args.K,
+                             flags=args.flags)
+                ev1.record(stream)
+                torch.cuda.synchronize()
+                e_ms += ev0.elapsed_time(ev1)
+                e_edges += m_sym if a == "cc" else m_reach[s]
+                if i == 0:
+                    h2d += o.numel() * 4 + c.numel() * 4 + (ww.numel() * 4 if ww is not None else 0)
+                    d2h += g.n * 4
+        e_max = allreduce([e_ms], tdist.ReduceOp.MAX if world > 1 else None, world)[0]
+        e_tot = allreduce([float(e_edges)], tdist.ReduceOp.SUM if world > 1 else None, world)[0]
+        e2e = {"value": e_tot / e_max / 1e6, "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h,
+               "how": "etg_run_host on pinned host CSR: H2D of off/col(/w), traversal, D2H of labels"}
+
+    # ---- CPU oracle baseline (rank 0, N = 1 only) ----
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        e, secs, sample = oracle_leg(args.config, algs, args.sources, 4242, budget_s=20.0, g=g, gs=gs)
+        cpu = {"value": e / secs / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"{sample} on {args.config} (single-threaded C oracle, {os.cpu_count()} host cores present)"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": max_ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": config_desc(args.config) + "; " + "+".join(algs) + " per step",
+                       "n": g.n, "m": g.m, "m_sym": m_sym, "K": args.K, "flags": args.flags,
+                       "sources": len(sources),
+                       "l2": "flushed (256 MiB write) before every traversal call; col/w 4 B x m each > 126 MB L2",
+                       "parallelism": f"{world} independent replica(s), own sources per rank"},
+            "per_alg": per_alg,
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": clk,
+        }
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.json_out:
+            with open(args.json_out, "w") as f:
+                f.write(s + "\n")
+    if world > 1:
+        tdist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

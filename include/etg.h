@@ -63,8 +63,10 @@ enum {
     ETG_NO_SMP = 1u << 2,      /* ablation: no shared-memory staging of neighbour segments */
     ETG_OFFSETS_U64 = 1u << 3, /* d_row_offsets holds uint64 (needed when m >= 2^32) */
     ETG_VALIDATE = 1u << 4,    /* etg_load_csr runs an O(n+m) device check of the CSR */
-    ETG_HOST_LOOP = 1u << 5    /* drive iterations from the host (count read back each
+    ETG_HOST_LOOP = 1u << 5,   /* drive iterations from the host (count read back each
                                   iteration) instead of a CUDA-graph conditional while node */
+    ETG_PROFILE = 1u << 6      /* implies ETG_HOST_LOOP; CUDA events around every scan and
+                                  expand launch on the handle's stream fill scan_ms/expand_ms */
 };
 
 typedef struct {
@@ -74,13 +76,17 @@ typedef struct {
 
 typedef struct {
     uint32_t iterations;       /* non-empty active sets processed (Proc. 1 while-loop trips) */
-    uint32_t reserved;
+    uint32_t expand_launches;  /* expand kernel launches (ETG_PROFILE) */
     uint64_t activations;      /* label improvements that won the atomic (incl. degree-0 vertices) */
+    uint64_t frontier_total;   /* sum over iterations of the active-set size */
     uint64_t shadows;          /* shadow vertices processed, summed over iterations (|N|, L152) */
     uint64_t edges_processed;  /* edges relaxed, summed over iterations */
     uint64_t vertices_reached; /* filled by etg_reach_stats */
     uint64_t edges_reached;    /* filled by etg_reach_stats: sum of out-degrees of reached vertices */
     float ms;                  /* device time of the traversal call (CUDA events) */
+    float scan_ms;             /* ETG_PROFILE: summed CUDA-event time of the udc_scan launches */
+    float expand_ms;           /* ETG_PROFILE: summed CUDA-event time of the expand launches */
+    float reserved;
 } etg_stats;
 
 /* Bytes of device workspace etg_load_csr needs for n vertices and m edges. */

@@ -23,11 +23,11 @@ import torch
 __all__ = [
     "EtgError", "Stats", "Graph", "load_csr", "csr_to_device", "to_u32_numpy",
     "run_host", "host_scratch_bytes", "kernel_launches", "lib",
-    "SYMMETRIC", "NO_UDC", "NO_SMP", "OFFSETS_U64", "VALIDATE", "HOST_LOOP",
+    "SYMMETRIC", "NO_UDC", "NO_SMP", "OFFSETS_U64", "VALIDATE", "HOST_LOOP", "PROFILE",
     "INF", "CAP", "BFS", "SSSP", "CC", "SSWP",
 ]
 
-SYMMETRIC, NO_UDC, NO_SMP, OFFSETS_U64, VALIDATE, HOST_LOOP = 1, 2, 4, 8, 16, 32
+SYMMETRIC, NO_UDC, NO_SMP, OFFSETS_U64, VALIDATE, HOST_LOOP, PROFILE = 1, 2, 4, 8, 16, 32, 64
 INF, CAP = 0xFFFFFFFF, 0xFFFFFFFE
 BFS, SSSP, CC, SSWP = 0, 1, 2, 3
 
@@ -46,10 +46,12 @@ class Options(ctypes.Structure):
 
 class Stats(ctypes.Structure):
     _fields_ = [
-        ("iterations", ctypes.c_uint32), ("reserved", ctypes.c_uint32),
-        ("activations", ctypes.c_uint64), ("shadows", ctypes.c_uint64),
-        ("edges_processed", ctypes.c_uint64), ("vertices_reached", ctypes.c_uint64),
-        ("edges_reached", ctypes.c_uint64), ("ms", ctypes.c_float),
+        ("iterations", ctypes.c_uint32), ("expand_launches", ctypes.c_uint32),
+        ("activations", ctypes.c_uint64), ("frontier_total", ctypes.c_uint64),
+        ("shadows", ctypes.c_uint64), ("edges_processed", ctypes.c_uint64),
+        ("vertices_reached", ctypes.c_uint64), ("edges_reached", ctypes.c_uint64),
+        ("ms", ctypes.c_float), ("scan_ms", ctypes.c_float), ("expand_ms", ctypes.c_float),
+        ("reserved", ctypes.c_float),
     ]
 
     def asdict(self):

@@ -114,6 +114,7 @@ struct etg_graph {
     int grid_init = 0;
     Ctl *h_ctl = nullptr;                 // pinned host mirror for readback
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    cudaEvent_t pev[3] = {nullptr, nullptr, nullptr};   // ETG_PROFILE: scan / expand brackets
     cudaGraphExec_t exec[4] = {nullptr, nullptr, nullptr, nullptr};
     cudaGraph_t graph[4] = {nullptr, nullptr, nullptr, nullptr};
 };
@@ -258,7 +259,10 @@ template <class OffT>
 etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stats *st) {
     Dev<OffT> d = make_dev<OffT>(g);
     cudaStream_t s = g->stream;
-    const bool host_loop = (g->flags & ETG_HOST_LOOP) != 0;
+    const bool profile = (g->flags & ETG_PROFILE) != 0;
+    const bool host_loop = profile || (g->flags & ETG_HOST_LOOP) != 0;
+    float scan_ms = 0.f, expand_ms = 0.f;
+    uint32_t expand_launches = 0;
     if (!host_loop) {
         etg_status rc = build_graph<OffT>(g, alg);
         if (rc != ETG_OK) return rc;
@@ -283,9 +287,12 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
         uint32_t it = 0;
         while (g->h_ctl->count[0] > 0) {
             void *scan_args[] = {&d};
+            if (profile) ETG_CU(cudaEventRecord(g->pev[0], s));
             ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+            if (profile) ETG_CU(cudaEventRecord(g->pev[1], s));
             void *exp_args[] = {&d, &cap_e};
             ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
+            if (profile) ETG_CU(cudaEventRecord(g->pev[2], s));
             void *adv_args[] = {&ctl, &none, &zero};
             ETG_CU(cudaLaunchKernel((const void *)advance_kernel, dim3(1), dim3(1), adv_args, 0, s));
             launches += 3;
@@ -293,6 +300,14 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
             // read back the size of the next active set ("actSet.isNotEmpty()", L207)
             ETG_CU(cudaMemcpyAsync(&g->h_ctl->count[0], &g->ctl->count[it & 1], 4, cudaMemcpyDeviceToHost, s));
             ETG_CU(cudaStreamSynchronize(s));
+            if (profile) {
+                float a = 0.f, b = 0.f;
+                ETG_CU(cudaEventElapsedTime(&a, g->pev[0], g->pev[1]));
+                ETG_CU(cudaEventElapsedTime(&b, g->pev[1], g->pev[2]));
+                scan_ms += a;
+                expand_ms += b;
+                ++expand_launches;
+            }
         }
     } else {
         ETG_CU(cudaGraphLaunch(g->exec[alg], s));
@@ -307,8 +322,12 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
         float ms = 0.f;
         ETG_CU(cudaEventElapsedTime(&ms, g->ev0, g->ev1));
         st->iterations = g->h_ctl->iterations;
-        st->reserved = 0;
+        st->expand_launches = expand_launches;
         st->activations = g->h_ctl->activations;
+        st->frontier_total = g->h_ctl->frontier;
+        st->scan_ms = scan_ms;
+        st->expand_ms = expand_ms;
+        st->reserved = 0.f;
         st->shadows = g->h_ctl->shadows;
         st->edges_processed = g->h_ctl->edges;
         st->vertices_reached = 0;
@@ -424,6 +443,8 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
         (e = cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess ||
         (e = cudaMallocHost(&g->h_ctl, sizeof(Ctl))) != cudaSuccess ||
         (e = cudaEventCreate(&g->ev0)) != cudaSuccess || (e = cudaEventCreate(&g->ev1)) != cudaSuccess ||
+        (e = cudaEventCreate(&g->pev[0])) != cudaSuccess || (e = cudaEventCreate(&g->pev[1])) != cudaSuccess ||
+        (e = cudaEventCreate(&g->pev[2])) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), g->stream)) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ws + L.stamp, 0, 4 * (n + 1), g->stream)) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ws + L.scan_status, 0, L.ctl - L.scan_status, g->stream)) != cudaSuccess) {
@@ -484,6 +505,8 @@ void etg_free(etg_graph *g) {
     }
     if (g->ev0) cudaEventDestroy(g->ev0);
     if (g->ev1) cudaEventDestroy(g->ev1);
+    for (int k = 0; k < 3; ++k)
+        if (g->pev[k]) cudaEventDestroy(g->pev[k]);
     if (g->h_ctl) cudaFreeHost(g->h_ctl);
     delete g;
 }

@@ -47,6 +47,7 @@ struct Ctl {
     unsigned long long activations;
     unsigned long long shadows;
     unsigned long long edges;
+    unsigned long long frontier;
     uint32_t *label;      // output label array of the current call
     uint32_t source;
     uint32_t error;       // ETG_VALIDATE result
@@ -157,6 +158,7 @@ __global__ void ctl_begin_kernel(Ctl *ctl, uint32_t *label, uint32_t source) {
     ctl->activations = 0;
     ctl->shadows = 0;
     ctl->edges = 0;
+    ctl->frontier = 0;
     ctl->label = label;
     ctl->source = source;
 }
@@ -488,6 +490,7 @@ __global__ __launch_bounds__(kBlock) void expand_kernel(Dev<OffT> d, uint32_t ca
 __global__ void advance_kernel(Ctl *ctl, cudaGraphConditionalHandle cond, int use_cond) {
     const uint32_t cur = ctl->iter & 1;
     if (ctl->count[cur] > 0) ctl->iterations += 1;
+    ctl->frontier += ctl->count[cur];
     ctl->shadows += ctl->nshadow;
     ctl->iter += 1;
     ctl->epoch += 1;
