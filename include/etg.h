@@ -123,10 +123,9 @@ etg_status etg_reach_stats(etg_graph *g, const uint32_t *d_label, uint32_t unrea
 
 /* Step A2 exposed for testing: the Unified Degree Cut of an active set, computed
  * by the same device code the traversal uses (Def. 3; Sec. IV-A).
- * d_active[n_active] (device) is the active set; every entry must have
- * out-degree >= 1 (degree-0 vertices produce no shadow and are filtered before
- * they reach the active set, L142).  Writes shadow q of the j-th active vertex
- * in active-set order as (d_id, d_start, d_end) = (v, off[v]+qK,
+ * d_active[n_active] (device) is the active set; degree-0 vertices produce no
+ * shadow (L142).  Writes shadow q of the j-th active vertex in active-set order
+ * as (d_id, d_start, d_end) = (v, off[v]+qK,
  * min(off[v]+(q+1)K, off[v+1])), uint32/uint64/uint64 device arrays of `cap`
  * entries; *n_out receives the number of shadows (ETG_ENOMEM if > cap). */
 etg_status etg_udc_slices(etg_graph *g, const uint32_t *d_active, uint32_t n_active,

@@ -12,6 +12,7 @@
 
 #include <atomic>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -46,6 +47,7 @@ struct Params {
     uint32_t ts;
     uint32_t ts_log2;
     bool udc;
+    bool idx;   // per-element owner index in shared memory (needs ts*K <= kCapE)
     bool smp;
     bool u64;
 };
@@ -64,14 +66,15 @@ Params derive(const etg_options *opt) {
         while (ts > 32 && ts * (uint64_t)p.K > kCapE) ts >>= 1;
         p.ts = ts;
     }
-    p.smp = p.udc && !(flags & ETG_NO_SMP) && (uint64_t)p.ts * p.K <= kCapE;
+    p.idx = p.udc && (uint64_t)p.ts * p.K <= kCapE;
+    p.smp = p.idx && !(flags & ETG_NO_SMP);
     p.ts_log2 = 0;
     while ((1u << p.ts_log2) < p.ts) ++p.ts_log2;
     return p;
 }
 
 struct Layout {
-    size_t F0, F1, S, tile_first, stamp, scan_status, ctl, total;
+    size_t R, F, B, D, S, tile_first, stamp, st_flag, st_agg, st_inc, ctl, total;
 };
 
 Layout layout(uint64_t n, uint64_t m, const Params &p) {
@@ -85,12 +88,16 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
     const uint64_t max_shadows = p.udc ? (m + p.K - 1) / p.K + n : n;   // sum ceil(d/K) <= m/K + |F|
     const uint64_t max_tiles = (max_shadows + p.ts - 1) / p.ts + 2;
     const uint64_t max_scan_tiles = (n + kScanTile - 1) / kScanTile + 2;
-    L.F0 = take(4 * (n + 1));
-    L.F1 = take(4 * (n + 1));
+    L.R = take(4 * (n + 1));
+    L.F = take(4 * (n + 1));
+    L.B = take((p.u64 ? 8 : 4) * (n + 1));
+    L.D = take(4 * (n + 1));
     L.S = take(4 * (n + 2));
     L.tile_first = take(4 * max_tiles);
     L.stamp = take(4 * (n + 1));
-    L.scan_status = take(8 * max_scan_tiles);
+    L.st_flag = take(4 * max_scan_tiles);
+    L.st_agg = take(8 * max_scan_tiles);
+    L.st_inc = take(8 * max_scan_tiles);
     L.ctl = take(sizeof(Ctl));
     L.total = o;
     return L;
@@ -110,6 +117,7 @@ struct etg_graph {
     Layout L{};
     Ctl *ctl = nullptr;
     int num_sms = 0;
+    uint32_t tune = 0;                    // ETG_TUNE (experiments only)
     int grid_scan = 0;
     int grid_init = 0;
     Ctl *h_ctl = nullptr;                 // pinned host mirror for readback
@@ -127,35 +135,41 @@ Dev<OffT> make_dev(const etg_graph *g) {
     d.off = static_cast<const OffT *>(g->off);
     d.col = g->col;
     d.w = g->w;
-    d.F[0] = reinterpret_cast<uint32_t *>(g->ws + g->L.F0);
-    d.F[1] = reinterpret_cast<uint32_t *>(g->ws + g->L.F1);
+    d.R = reinterpret_cast<uint32_t *>(g->ws + g->L.R);
+    d.F = reinterpret_cast<uint32_t *>(g->ws + g->L.F);
+    d.B = reinterpret_cast<OffT *>(g->ws + g->L.B);
+    d.D = reinterpret_cast<uint32_t *>(g->ws + g->L.D);
     d.S = reinterpret_cast<uint32_t *>(g->ws + g->L.S);
     d.tile_first = reinterpret_cast<uint32_t *>(g->ws + g->L.tile_first);
     d.stamp = reinterpret_cast<uint32_t *>(g->ws + g->L.stamp);
-    d.scan_status = reinterpret_cast<unsigned long long *>(g->ws + g->L.scan_status);
+    d.st_flag = reinterpret_cast<uint32_t *>(g->ws + g->L.st_flag);
+    d.st_agg = reinterpret_cast<unsigned long long *>(g->ws + g->L.st_agg);
+    d.st_inc = reinterpret_cast<unsigned long long *>(g->ws + g->L.st_inc);
     d.ctl = g->ctl;
     d.n = (uint32_t)g->n;
     d.K = g->p.K;
     d.ts = g->p.ts;
     d.ts_log2 = g->p.ts_log2;
+    d.tune = g->tune;
     return d;
 }
 
 // --- kernel selection ------------------------------------------------------ //
 template <class OffT, int ALG>
-const void *expand_fn(bool udc, bool smp) {
-    if (!udc) return (const void *)expand_kernel<OffT, ALG, false, false>;
-    if (smp) return (const void *)expand_kernel<OffT, ALG, true, true>;
-    return (const void *)expand_kernel<OffT, ALG, true, false>;
+const void *expand_fn(bool udc, bool idx, bool smp) {
+    if (!udc) return (const void *)expand_kernel<OffT, ALG, false, false, false>;
+    if (smp) return (const void *)expand_kernel<OffT, ALG, true, true, true>;
+    if (idx) return (const void *)expand_kernel<OffT, ALG, true, true, false>;
+    return (const void *)expand_kernel<OffT, ALG, true, false, false>;
 }
 
 template <class OffT>
-const void *expand_fn_alg(int alg, bool udc, bool smp) {
+const void *expand_fn_alg(int alg, bool udc, bool idx, bool smp) {
     switch (alg) {
-        case ALG_BFS: return expand_fn<OffT, ALG_BFS>(udc, smp);
-        case ALG_SSSP: return expand_fn<OffT, ALG_SSSP>(udc, smp);
-        case ALG_CC: return expand_fn<OffT, ALG_CC>(udc, smp);
-        default: return expand_fn<OffT, ALG_SSWP>(udc, smp);
+        case ALG_BFS: return expand_fn<OffT, ALG_BFS>(udc, idx, smp);
+        case ALG_SSSP: return expand_fn<OffT, ALG_SSSP>(udc, idx, smp);
+        case ALG_CC: return expand_fn<OffT, ALG_CC>(udc, idx, smp);
+        default: return expand_fn<OffT, ALG_SSWP>(udc, idx, smp);
     }
 }
 
@@ -170,15 +184,15 @@ const void *init_fn(int alg) {
 }
 
 template <class OffT>
-const void *scan_fn(bool udc) {
+const void *scan_fn(bool udc, int) {
     return udc ? (const void *)udc_scan_kernel<OffT, true> : (const void *)udc_scan_kernel<OffT, false>;
 }
 
 size_t expand_smem(const Params &p, int alg) {
-    if (!p.smp) return 0;
+    if (!p.idx) return 0;
     const size_t cap = (size_t)p.ts * p.K;
     const bool kw = (alg == ALG_SSSP || alg == ALG_SSWP);
-    return cap * 4 * (kw ? 2 : 1) + cap;
+    return (p.smp ? cap * 4 * (kw ? 2 : 1) : 0) + cap;
 }
 
 struct Launch {
@@ -189,9 +203,10 @@ struct Launch {
 
 template <class OffT>
 etg_status expand_launch(etg_graph *g, int alg, Launch &out) {
-    out.fn = expand_fn_alg<OffT>(alg, g->p.udc, g->p.smp);
+    out.fn = expand_fn_alg<OffT>(alg, g->p.udc, g->p.idx, g->p.smp);
     out.smem = expand_smem(g->p, alg);
     ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)out.smem));
+    ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
     int nb = 0;
     ETG_CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, out.fn, kBlock, out.smem));
     if (nb < 1) nb = 1;
@@ -225,7 +240,7 @@ etg_status build_graph(etg_graph *g, int alg) {
     cudaGraphNode_t n_scan, n_exp, n_adv;
     void *scan_args[] = {&d};
     memset(&kp, 0, sizeof(kp));
-    kp.func = const_cast<void *>(scan_fn<OffT>(g->p.udc));
+    kp.func = const_cast<void *>(scan_fn<OffT>(g->p.udc, alg));
     kp.gridDim = dim3(g->grid_scan);
     kp.blockDim = dim3(kBlock);
     kp.kernelParams = scan_args;
@@ -288,7 +303,7 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
         while (g->h_ctl->count[0] > 0) {
             void *scan_args[] = {&d};
             if (profile) ETG_CU(cudaEventRecord(g->pev[0], s));
-            ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+            ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
             if (profile) ETG_CU(cudaEventRecord(g->pev[1], s));
             void *exp_args[] = {&d, &cap_e};
             ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
@@ -378,8 +393,9 @@ etg_status udc_impl(etg_graph *g, const uint32_t *act, uint32_t n_act, uint32_t 
     Dev<OffT> d = make_dev<OffT>(g);
     cudaStream_t s = g->stream;
     ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, nullptr, 0);
-    if (n_act) ETG_CU(cudaMemcpyAsync(d.F[0], act, 4ull * n_act, cudaMemcpyDeviceToDevice, s));
-    ETG_CU(cudaMemcpyAsync(&g->ctl->count[0], &n_act, 4, cudaMemcpyHostToDevice, s));
+    if (n_act) ETG_CU(cudaMemcpyAsync(d.R, act, 4ull * n_act, cudaMemcpyDeviceToDevice, s));
+    g->h_ctl->count[0] = n_act;
+    ETG_CU(cudaMemcpyAsync(&g->ctl->count[0], &g->h_ctl->count[0], 4, cudaMemcpyHostToDevice, s));
     udc_scan_kernel<OffT, true><<<g->grid_scan, kBlock, 0, s>>>(d);
     ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     ETG_CU(cudaStreamSynchronize(s));
@@ -447,9 +463,10 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
         (e = cudaEventCreate(&g->pev[2])) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), g->stream)) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ws + L.stamp, 0, 4 * (n + 1), g->stream)) != cudaSuccess ||
-        (e = cudaMemsetAsync(g->ws + L.scan_status, 0, L.ctl - L.scan_status, g->stream)) != cudaSuccess) {
+        (e = cudaMemsetAsync(g->ws + L.st_flag, 0, L.st_agg - L.st_flag, g->stream)) != cudaSuccess) {
         return bail(fail(ETG_ECUDA, std::string("load: ") + cudaGetErrorString(e)));
     }
+    if (const char *t = getenv("ETG_TUNE")) g->tune = (uint32_t)strtoul(t, nullptr, 0);
     g->grid_scan = g->num_sms * 2;
     g->grid_init = g->num_sms * 8;
     if (flags & ETG_VALIDATE) {

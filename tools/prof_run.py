@@ -1,0 +1,35 @@
+"""Minimal driver for ncu captures: build a config, run one traversal per algorithm
+in host-loop mode (ETG_HOST_LOOP, so every kernel is a host launch ncu can see)."""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+import graphgen as gg  # noqa: E402
+import paper_conf_ipps_wangzlg19_b200 as etg  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", default="C2")
+ap.add_argument("--algs", default="bfs")
+ap.add_argument("--K", type=int, default=32)
+ap.add_argument("--flags", type=int, default=etg.HOST_LOOP)
+ap.add_argument("--repeat", type=int, default=1)
+a = ap.parse_args()
+dev = torch.device("cuda:0")
+algs = a.algs.split(",")
+g = gg.make(a.config, device=dev, weights="sssp" in algs)
+src = gg.sample_sources(g, 1, 4242)[0]
+o, c, w, fl = etg.csr_to_device(g.off, g.col, g.w, device=dev)
+G = etg.Graph(o, c, w, n=g.n, K=a.K, flags=a.flags | fl)
+for _ in range(a.repeat):
+    for alg in algs:
+        if alg == "cc":
+            gs = gg.make(a.config, device=dev, symmetric=True, weights=False)
+            o2, c2, _, fl2 = etg.csr_to_device(gs.off, gs.col, None, device=dev)
+            Gs = etg.Graph(o2, c2, None, n=gs.n, K=a.K, flags=a.flags | fl2, symmetric=True)
+            _, st = Gs.cc()
+        else:
+            _, st = G.run({"bfs": etg.BFS, "sssp": etg.SSSP, "sswp": etg.SSWP}[alg], src)
+        print(alg, st.asdict())
