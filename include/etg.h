@@ -77,7 +77,8 @@ typedef struct {
 typedef struct {
     uint32_t iterations;       /* non-empty active sets processed (Proc. 1 while-loop trips) */
     uint32_t expand_launches;  /* expand kernel launches (ETG_PROFILE) */
-    uint64_t activations;      /* label improvements that won the atomic (incl. degree-0 vertices) */
+    uint64_t activations;      /* vertex activations: (vertex, iteration) pairs marked active,
+                                  the initial active set included (degree-0 vertices too) */
     uint64_t frontier_total;   /* sum over iterations of the active-set size */
     uint64_t shadows;          /* shadow vertices processed, summed over iterations (|N|, L152) */
     uint64_t edges_processed;  /* edges relaxed, summed over iterations */
@@ -123,14 +124,25 @@ etg_status etg_reach_stats(etg_graph *g, const uint32_t *d_label, uint32_t unrea
 
 /* Step A2 exposed for testing: the Unified Degree Cut of an active set, computed
  * by the same device code the traversal uses (Def. 3; Sec. IV-A).
- * d_active[n_active] (device) is the active set; degree-0 vertices produce no
- * shadow (L142).  Writes shadow q of the j-th active vertex in active-set order
- * as (d_id, d_start, d_end) = (v, off[v]+qK,
+ * d_active[n_active] (device) is the active set (a set: duplicates are merged);
+ * degree-0 vertices produce no shadow (L142).  Active vertices are taken in
+ * increasing id order (the library keeps the active set as a bitmap); shadow q
+ * of vertex v is written as (d_id, d_start, d_end) = (v, off[v]+qK,
  * min(off[v]+(q+1)K, off[v+1])), uint32/uint64/uint64 device arrays of `cap`
  * entries; *n_out receives the number of shadows (ETG_ENOMEM if > cap). */
 etg_status etg_udc_slices(etg_graph *g, const uint32_t *d_active, uint32_t n_active,
                           uint32_t *d_id, uint64_t *d_start, uint64_t *d_end,
                           uint64_t cap, uint64_t *n_out);
+
+/* Tuning/debug: run `alg` from `source` until the active set of iteration
+ * `depth` is ready, snapshot it, then time `reps` launches of the expand kernel
+ * on that same state (labels restored from d_saved, n words of device scratch,
+ * before each launch).  tune = experiment bits (0 = the production kernel).
+ * Outputs the mean launch time, the edges one launch relaxes and the active-set
+ * size.  Not part of the traversal path; d_label is left as the snapshot. */
+etg_status etg_debug_expand_replay(etg_graph *g, int alg, uint32_t source, uint32_t depth,
+                                   uint32_t tune, int reps, uint32_t *d_label, uint32_t *d_saved,
+                                   float *ms, uint64_t *edges, uint32_t *n_active);
 
 /* Release a handle (does not free the borrowed device memory). */
 void etg_free(etg_graph *g);

@@ -32,7 +32,7 @@ INF, CAP = 0xFFFFFFFF, 0xFFFFFFFE
 BFS, SSSP, CC, SSWP = 0, 1, 2, 3
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_LIB_PATH = os.path.join(_HERE, "libetg.so")
+_LIB_PATH = os.environ.get("ETG_LIB_PATH") or os.path.join(_HERE, "libetg.so")
 _lib = None
 
 
@@ -82,6 +82,9 @@ def lib():
             "etg_status_str": (ctypes.c_char_p, [st]),
             "etg_last_error": (ctypes.c_char_p, []),
             "etg_kernel_launches": (u64, []),
+            "etg_debug_expand_replay": (st, [p, ctypes.c_int, u32, u32, u32, ctypes.c_int, p, p,
+                                             ctypes.POINTER(ctypes.c_float), ctypes.POINTER(u64),
+                                             ctypes.POINTER(u32)]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -248,6 +251,16 @@ class Graph:
         _check(L.etg_udc_slices(self._h, _ptr(active), n_act, _ptr(ids), _ptr(st), _ptr(en),
                                 cnt, ctypes.byref(out)), "etg_udc_slices")
         return ids[:cnt], st[:cnt], en[:cnt]
+
+    def debug_expand_replay(self, alg: int, source: int, depth: int, tune: int = 0, reps: int = 5):
+        """Time the expand kernel on the snapshot of iteration `depth` (tuning aid)."""
+        lab = torch.empty(self.n, dtype=torch.int32, device=self.device)
+        saved = torch.empty(self.n, dtype=torch.int32, device=self.device)
+        ms, edges, nact = ctypes.c_float(), ctypes.c_uint64(), ctypes.c_uint32()
+        _check(lib().etg_debug_expand_replay(self._h, alg, source, depth, tune, reps, _ptr(lab),
+                                             _ptr(saved), ctypes.byref(ms), ctypes.byref(edges),
+                                             ctypes.byref(nact)), "etg_debug_expand_replay")
+        return ms.value, int(edges.value), int(nact.value)
 
     def close(self):
         if getattr(self, "_h", None):

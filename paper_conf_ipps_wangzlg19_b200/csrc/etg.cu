@@ -2,12 +2,12 @@
 //
 // The engine owns nothing on the device: the CSR and a caller-provided
 // workspace are borrowed (etg_load_csr).  Per traversal call it enqueues, on the
-// handle's stream: ctl_begin + init (A1), then the Proc. 1 while-loop
-// as a CUDA graph with a conditional WHILE node whose body is
-// udc_scan -> expand -> advance (A2-A6).  The loop condition is set on the
-// device, so the host synchronises once per call, not once per iteration.
-// ETG_HOST_LOOP replaces the graph by a host loop that reads the active-set
-// size back every iteration (the paper's own control flow).
+// handle's stream: ctl_begin + init (A1) and the first udc_scan, then the
+// Proc. 1 while-loop as a CUDA graph with a conditional WHILE
+// node whose body is expand -> udc_scan (A2-A6); the scan's last tile sets the
+// loop condition on the device, so the host synchronises once per call, not
+// once per iteration.  ETG_HOST_LOOP replaces the graph by a host loop that
+// reads the active-set size back every iteration (the paper's own control flow).
 #include <cuda_runtime.h>
 
 #include <atomic>
@@ -24,6 +24,11 @@ using namespace etg;
 namespace {
 
 thread_local std::string g_err;
+
+uint32_t env_tune() {
+    const char *t = getenv("ETG_TUNE");
+    return t ? (uint32_t)strtoul(t, nullptr, 0) : 0u;
+}
 std::atomic<uint64_t> g_launches{0};
 
 etg_status fail(etg_status s, const std::string &msg) {
@@ -47,13 +52,15 @@ struct Params {
     uint32_t ts;
     uint32_t ts_log2;
     bool udc;
+    bool warp;  // warp-centric expand (ts = 32, registers only); else the CTA-tile kernel
     bool idx;   // per-element owner index in shared memory (needs ts*K <= kCapE)
     bool smp;
     bool u64;
 };
 
-Params derive(const etg_options *opt) {
+Params derive(const etg_options *opt, uint32_t tune) {
     Params p;
+    p.warp = !(tune & 2u);
     const uint32_t flags = opt ? opt->flags : 0u;
     p.K = (opt && opt->degree_limit_k) ? opt->degree_limit_k : 32u;
     p.udc = !(flags & ETG_NO_UDC);
@@ -68,13 +75,18 @@ Params derive(const etg_options *opt) {
     }
     p.idx = p.udc && (uint64_t)p.ts * p.K <= kCapE;
     p.smp = p.idx && !(flags & ETG_NO_SMP);
+    if (p.warp) {
+        p.ts = 32;
+        p.idx = p.smp = false;
+    }
     p.ts_log2 = 0;
     while ((1u << p.ts_log2) < p.ts) ++p.ts_log2;
     return p;
 }
 
 struct Layout {
-    size_t R, F, B, D, S, tile_first, stamp, st_flag, st_agg, st_inc, ctl, total;
+    size_t Q, F, B, D, S, tile_first, st_flag, st_agg, st_inc, ctl, total;
+    uint32_t nwords;
 };
 
 Layout layout(uint64_t n, uint64_t m, const Params &p) {
@@ -86,15 +98,16 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
         return at;
     };
     const uint64_t max_shadows = p.udc ? (m + p.K - 1) / p.K + n : n;   // sum ceil(d/K) <= m/K + |F|
-    const uint64_t max_tiles = (max_shadows + p.ts - 1) / p.ts + 2;
-    const uint64_t max_scan_tiles = (n + kScanTile - 1) / kScanTile + 2;
-    L.R = take(4 * (n + 1));
+    const uint64_t max_tiles = (max_shadows + 31) / 32 + 2;      // sized for the smallest tile (32)
+    const uint64_t max_scan_tiles = ((n + 31) / 32 + kScanTile - 1) / kScanTile + 2;
+    const uint64_t words = (n + 31) / 32;
+    L.nwords = (uint32_t)((words + kScanWords - 1) / kScanWords * kScanWords);
+    L.Q = take(4ull * L.nwords);
     L.F = take(4 * (n + 1));
     L.B = take((p.u64 ? 8 : 4) * (n + 1));
     L.D = take(4 * (n + 1));
     L.S = take(4 * (n + 2));
     L.tile_first = take(4 * max_tiles);
-    L.stamp = take(4 * (n + 1));
     L.st_flag = take(4 * max_scan_tiles);
     L.st_agg = take(8 * max_scan_tiles);
     L.st_inc = take(8 * max_scan_tiles);
@@ -135,13 +148,13 @@ Dev<OffT> make_dev(const etg_graph *g) {
     d.off = static_cast<const OffT *>(g->off);
     d.col = g->col;
     d.w = g->w;
-    d.R = reinterpret_cast<uint32_t *>(g->ws + g->L.R);
+    d.Q = reinterpret_cast<uint32_t *>(g->ws + g->L.Q);
+    d.nwords = g->L.nwords;
     d.F = reinterpret_cast<uint32_t *>(g->ws + g->L.F);
     d.B = reinterpret_cast<OffT *>(g->ws + g->L.B);
     d.D = reinterpret_cast<uint32_t *>(g->ws + g->L.D);
     d.S = reinterpret_cast<uint32_t *>(g->ws + g->L.S);
     d.tile_first = reinterpret_cast<uint32_t *>(g->ws + g->L.tile_first);
-    d.stamp = reinterpret_cast<uint32_t *>(g->ws + g->L.stamp);
     d.st_flag = reinterpret_cast<uint32_t *>(g->ws + g->L.st_flag);
     d.st_agg = reinterpret_cast<unsigned long long *>(g->ws + g->L.st_agg);
     d.st_inc = reinterpret_cast<unsigned long long *>(g->ws + g->L.st_inc);
@@ -163,8 +176,21 @@ const void *expand_fn(bool udc, bool idx, bool smp) {
     return (const void *)expand_kernel<OffT, ALG, true, false, false>;
 }
 
+template <class OffT, int ALG>
+const void *expand_warp_fn(bool udc) {
+    return udc ? (const void *)expand_warp_kernel<OffT, ALG, true> : (const void *)expand_warp_kernel<OffT, ALG, false>;
+}
+
 template <class OffT>
-const void *expand_fn_alg(int alg, bool udc, bool idx, bool smp) {
+const void *expand_fn_alg(int alg, bool udc, bool idx, bool smp, bool warp) {
+    if (warp) {
+        switch (alg) {
+            case ALG_BFS: return expand_warp_fn<OffT, ALG_BFS>(udc);
+            case ALG_SSSP: return expand_warp_fn<OffT, ALG_SSSP>(udc);
+            case ALG_CC: return expand_warp_fn<OffT, ALG_CC>(udc);
+            default: return expand_warp_fn<OffT, ALG_SSWP>(udc);
+        }
+    }
     switch (alg) {
         case ALG_BFS: return expand_fn<OffT, ALG_BFS>(udc, idx, smp);
         case ALG_SSSP: return expand_fn<OffT, ALG_SSSP>(udc, idx, smp);
@@ -184,8 +210,10 @@ const void *init_fn(int alg) {
 }
 
 template <class OffT>
-const void *scan_fn(bool udc, int) {
-    return udc ? (const void *)udc_scan_kernel<OffT, true> : (const void *)udc_scan_kernel<OffT, false>;
+const void *scan_fn(bool udc, int alg) {
+    if (alg == ALG_BFS)
+        return udc ? (const void *)udc_scan_kernel<OffT, true, true> : (const void *)udc_scan_kernel<OffT, false, true>;
+    return udc ? (const void *)udc_scan_kernel<OffT, true, false> : (const void *)udc_scan_kernel<OffT, false, false>;
 }
 
 size_t expand_smem(const Params &p, int alg) {
@@ -203,8 +231,8 @@ struct Launch {
 
 template <class OffT>
 etg_status expand_launch(etg_graph *g, int alg, Launch &out) {
-    out.fn = expand_fn_alg<OffT>(alg, g->p.udc, g->p.idx, g->p.smp);
-    out.smem = expand_smem(g->p, alg);
+    out.fn = expand_fn_alg<OffT>(alg, g->p.udc, g->p.idx, g->p.smp, g->p.warp);
+    out.smem = g->p.warp ? 0 : expand_smem(g->p, alg);
     ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)out.smem));
     ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
     int nb = 0;
@@ -237,33 +265,25 @@ etg_status build_graph(etg_graph *g, int alg) {
     cudaGraph_t body = cp.conditional.phGraph_out[0];
 
     cudaKernelNodeParams kp;
-    cudaGraphNode_t n_scan, n_exp, n_adv;
-    void *scan_args[] = {&d};
-    memset(&kp, 0, sizeof(kp));
-    kp.func = const_cast<void *>(scan_fn<OffT>(g->p.udc, alg));
-    kp.gridDim = dim3(g->grid_scan);
-    kp.blockDim = dim3(kBlock);
-    kp.kernelParams = scan_args;
-    ETG_CU(cudaGraphAddKernelNode(&n_scan, body, nullptr, 0, &kp));
-
+    cudaGraphNode_t n_scan, n_exp;
     void *exp_args[] = {&d, &cap_e};
     memset(&kp, 0, sizeof(kp));
+    if (g->p.warp) exp_args[1] = nullptr;
     kp.func = const_cast<void *>(ex.fn);
     kp.gridDim = ex.grid;
     kp.blockDim = dim3(kBlock);
     kp.sharedMemBytes = (unsigned)ex.smem;
     kp.kernelParams = exp_args;
-    ETG_CU(cudaGraphAddKernelNode(&n_exp, body, &n_scan, 1, &kp));
+    ETG_CU(cudaGraphAddKernelNode(&n_exp, body, nullptr, 0, &kp));
 
-    Ctl *ctl = g->ctl;
     int use_cond = 1;
-    void *adv_args[] = {&ctl, &cond, &use_cond};
+    void *scan_args[] = {&d, &cond, &use_cond};
     memset(&kp, 0, sizeof(kp));
-    kp.func = (void *)advance_kernel;
-    kp.gridDim = dim3(1);
-    kp.blockDim = dim3(1);
-    kp.kernelParams = adv_args;
-    ETG_CU(cudaGraphAddKernelNode(&n_adv, body, &n_exp, 1, &kp));
+    kp.func = const_cast<void *>(scan_fn<OffT>(g->p.udc, alg));
+    kp.gridDim = dim3(g->grid_scan);
+    kp.blockDim = dim3(kBlock);
+    kp.kernelParams = scan_args;
+    ETG_CU(cudaGraphAddKernelNode(&n_scan, body, &n_exp, 1, &kp));
 
     ETG_CU(cudaGraphInstantiate(&g->exec[alg], graph, 0));
     g->graph[alg] = graph;
@@ -288,39 +308,37 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
         void *args[] = {&d, &label, &source};
         ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), args, 0, s));
     }
-    uint64_t launches = 2;
+    cudaGraphConditionalHandle none = 0;
+    int zero = 0;
+    void *scan_args[] = {&d, &none, &zero};
+    // A2 of the initial active set (Proc. 1 "Init actSet")
+    ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+    uint64_t launches = 3;
     if (host_loop) {
         Launch ex;
         etg_status rc = expand_launch<OffT>(g, alg, ex);
         if (rc != ETG_OK) return rc;
         uint32_t cap_e = g->p.ts * g->p.K;
-        cudaGraphConditionalHandle none = 0;
-        int zero = 0;
-        Ctl *ctl = g->ctl;
-        ETG_CU(cudaMemcpyAsync(&g->h_ctl->count[0], &g->ctl->count[0], 4, cudaMemcpyDeviceToHost, s));
-        ETG_CU(cudaStreamSynchronize(s));
-        uint32_t it = 0;
-        while (g->h_ctl->count[0] > 0) {
-            void *scan_args[] = {&d};
-            if (profile) ETG_CU(cudaEventRecord(g->pev[0], s));
-            ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
-            if (profile) ETG_CU(cudaEventRecord(g->pev[1], s));
-            void *exp_args[] = {&d, &cap_e};
-            ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
-            if (profile) ETG_CU(cudaEventRecord(g->pev[2], s));
-            void *adv_args[] = {&ctl, &none, &zero};
-            ETG_CU(cudaLaunchKernel((const void *)advance_kernel, dim3(1), dim3(1), adv_args, 0, s));
-            launches += 3;
-            ++it;
-            // read back the size of the next active set ("actSet.isNotEmpty()", L207)
-            ETG_CU(cudaMemcpyAsync(&g->h_ctl->count[0], &g->ctl->count[it & 1], 4, cudaMemcpyDeviceToHost, s));
+        void *exp_args[] = {&d, &cap_e};
+        if (g->p.warp) exp_args[1] = nullptr;
+        for (;;) {
+            // "while actSet.isNotEmpty()" (L207): read the compacted size back
+            ETG_CU(cudaMemcpyAsync(&g->h_ctl->nF, &g->ctl->nF, 4, cudaMemcpyDeviceToHost, s));
             ETG_CU(cudaStreamSynchronize(s));
+            if (g->h_ctl->nF == 0) break;
+            if (profile) ETG_CU(cudaEventRecord(g->pev[0], s));
+            ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
+            if (profile) ETG_CU(cudaEventRecord(g->pev[1], s));
+            ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+            if (profile) ETG_CU(cudaEventRecord(g->pev[2], s));
+            launches += 2;
             if (profile) {
+                ETG_CU(cudaEventSynchronize(g->pev[2]));
                 float a = 0.f, b = 0.f;
                 ETG_CU(cudaEventElapsedTime(&a, g->pev[0], g->pev[1]));
                 ETG_CU(cudaEventElapsedTime(&b, g->pev[1], g->pev[2]));
-                scan_ms += a;
-                expand_ms += b;
+                expand_ms += a;
+                scan_ms += b;
                 ++expand_launches;
             }
         }
@@ -331,7 +349,7 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
     ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     ETG_CU(cudaStreamSynchronize(s));
     ETG_CU(cudaGetLastError());
-    if (!host_loop) launches += 3ull * g->h_ctl->iter;
+    if (!host_loop) launches += 2ull * g->h_ctl->depth;   // body runs = scans after the first
     g_launches += launches;
     if (st) {
         float ms = 0.f;
@@ -393,16 +411,80 @@ etg_status udc_impl(etg_graph *g, const uint32_t *act, uint32_t n_act, uint32_t 
     Dev<OffT> d = make_dev<OffT>(g);
     cudaStream_t s = g->stream;
     ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, nullptr, 0);
-    if (n_act) ETG_CU(cudaMemcpyAsync(d.R, act, 4ull * n_act, cudaMemcpyDeviceToDevice, s));
-    g->h_ctl->count[0] = n_act;
-    ETG_CU(cudaMemcpyAsync(&g->ctl->count[0], &g->h_ctl->count[0], 4, cudaMemcpyHostToDevice, s));
-    udc_scan_kernel<OffT, true><<<g->grid_scan, kBlock, 0, s>>>(d);
+    if (n_act) mark_kernel<<<g->num_sms, kBlock, 0, s>>>(d.Q, act, n_act);
+    udc_scan_kernel<OffT, true, false><<<g->grid_scan, kBlock, 0, s>>>(d, 0, 0);
     ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     ETG_CU(cudaStreamSynchronize(s));
     *n_out = g->h_ctl->nshadow;
     if (g->h_ctl->nshadow > cap) return fail(ETG_ENOMEM, "cap too small for the shadow list");
     udc_dump_kernel<OffT, true><<<g->num_sms * 4, kBlock, 0, s>>>(d, id, start, end);
     g_launches += 3;
+    ETG_CU(cudaStreamSynchronize(s));
+    ETG_CU(cudaGetLastError());
+    return ETG_OK;
+}
+
+// Debug/tuning: advance a traversal to the active set of `depth`, snapshot the
+// state, then time `reps` launches of the expand kernel on that same state with
+// the given tune bits (labels and the bitmap restored before every launch).
+template <class OffT>
+etg_status replay_impl(etg_graph *g, int alg, uint32_t source, uint32_t depth, uint32_t tune, int reps,
+                       uint32_t *label, uint32_t *saved, float *ms_out, uint64_t *edges_out,
+                       uint32_t *nF_out) {
+    Dev<OffT> d = make_dev<OffT>(g);
+    cudaStream_t s = g->stream;
+    Launch ex;
+    etg_status rc = expand_launch<OffT>(g, alg, ex);
+    if (rc != ETG_OK) return rc;
+    uint32_t cap_e = g->p.ts * g->p.K;
+    void *exp_args[] = {&d, &cap_e};
+    if (g->p.warp) exp_args[1] = nullptr;
+    cudaGraphConditionalHandle none = 0;
+    int zero = 0;
+    void *scan_args[] = {&d, &none, &zero};
+    ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, label, source);
+    void *iargs[] = {&d, &label, &source};
+    ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), iargs, 0, s));
+    ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+    for (;;) {
+        ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+        ETG_CU(cudaStreamSynchronize(s));
+        if (g->h_ctl->depth >= depth || g->h_ctl->nF == 0) break;
+        ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
+        ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+    }
+    ETG_CU(cudaMemsetAsync(&g->ctl->reached_v, 0, 8, s));
+    ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    ETG_CU(cudaStreamSynchronize(s));
+    const Ctl snap = *g->h_ctl;
+    *nF_out = snap.nF;
+    ETG_CU(cudaMemcpyAsync(saved, label, 4ull * g->n, cudaMemcpyDeviceToDevice, s));
+    Dev<OffT> dt = d;
+    dt.tune = tune;
+    void *targs[] = {&dt, &cap_e};
+    if (g->p.warp) targs[1] = nullptr;
+    float total = 0.f;
+    for (int r = 0; r < reps; ++r) {
+        ETG_CU(cudaMemcpyAsync(label, saved, 4ull * g->n, cudaMemcpyDeviceToDevice, s));
+        ETG_CU(cudaMemsetAsync(d.Q, 0, 4ull * g->L.nwords, s));
+        *g->h_ctl = snap;
+        ETG_CU(cudaMemcpyAsync(g->ctl, g->h_ctl, sizeof(Ctl), cudaMemcpyHostToDevice, s));
+        ETG_CU(cudaEventRecord(g->pev[0], s));
+        ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), targs, ex.smem, s));
+        ETG_CU(cudaEventRecord(g->pev[1], s));
+        ETG_CU(cudaEventSynchronize(g->pev[1]));
+        float ms = 0.f;
+        ETG_CU(cudaEventElapsedTime(&ms, g->pev[0], g->pev[1]));
+        total += ms;
+    }
+    ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    ETG_CU(cudaStreamSynchronize(s));
+    *edges_out = g->h_ctl->edges - snap.edges;
+    if (tune & 32u) *nF_out = (uint32_t)(g->h_ctl->reached_v / (reps ? reps : 1));   // passes
+    *ms_out = reps ? total / reps : 0.f;
+    // leave the handle consistent: labels restored, bitmap clear
+    ETG_CU(cudaMemcpyAsync(label, saved, 4ull * g->n, cudaMemcpyDeviceToDevice, s));
+    ETG_CU(cudaMemsetAsync(d.Q, 0, 4ull * g->L.nwords, s));
     ETG_CU(cudaStreamSynchronize(s));
     ETG_CU(cudaGetLastError());
     return ETG_OK;
@@ -416,7 +498,7 @@ etg_status udc_impl(etg_graph *g, const uint32_t *act, uint32_t n_act, uint32_t 
 extern "C" {
 
 size_t etg_workspace_bytes(uint64_t n, uint64_t m, const etg_options *opt) {
-    return layout(n, m, derive(opt)).total;
+    return layout(n, m, derive(opt, env_tune())).total;
 }
 
 etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_row_offsets,
@@ -425,7 +507,8 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
     if (!out) return fail(ETG_EINVAL, "out is NULL");
     *out = nullptr;
     if (!d_row_offsets || (m && !d_col_idx) || !d_workspace) return fail(ETG_EINVAL, "NULL device pointer");
-    const Params p = derive(opt);
+    const uint32_t tune = env_tune();
+    const Params p = derive(opt, tune);
     const uint32_t flags = opt ? opt->flags : 0u;
     if (n > 0xFFFFFFFEull) return fail(ETG_ERANGE, "n > 2^32 - 2");
     if (!p.u64 && m > 0xFFFFFFFFull) return fail(ETG_ERANGE, "m >= 2^32 needs ETG_OFFSETS_U64");
@@ -462,11 +545,11 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
         (e = cudaEventCreate(&g->pev[0])) != cudaSuccess || (e = cudaEventCreate(&g->pev[1])) != cudaSuccess ||
         (e = cudaEventCreate(&g->pev[2])) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), g->stream)) != cudaSuccess ||
-        (e = cudaMemsetAsync(g->ws + L.stamp, 0, 4 * (n + 1), g->stream)) != cudaSuccess ||
+        (e = cudaMemsetAsync(g->ws + L.Q, 0, 4ull * L.nwords, g->stream)) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ws + L.st_flag, 0, L.st_agg - L.st_flag, g->stream)) != cudaSuccess) {
         return bail(fail(ETG_ECUDA, std::string("load: ") + cudaGetErrorString(e)));
     }
-    if (const char *t = getenv("ETG_TUNE")) g->tune = (uint32_t)strtoul(t, nullptr, 0);
+    g->tune = tune;
     g->grid_scan = g->num_sms * 2;
     g->grid_init = g->num_sms * 8;
     if (flags & ETG_VALIDATE) {
@@ -514,6 +597,16 @@ etg_status etg_udc_slices(etg_graph *g, const uint32_t *d_active, uint32_t n_act
                     : udc_impl<uint32_t>(g, d_active, n_active, d_id, d_start, d_end, cap, n_out);
 }
 
+etg_status etg_debug_expand_replay(etg_graph *g, int alg, uint32_t source, uint32_t depth, uint32_t tune,
+                                   int reps, uint32_t *d_label, uint32_t *d_saved, float *ms,
+                                   uint64_t *edges, uint32_t *n_active) {
+    if (!g || !d_label || !d_saved || !ms || !edges || !n_active) return fail(ETG_EINVAL, "NULL argument");
+    if (alg < 0 || alg > 3) return fail(ETG_EINVAL, "alg must be 0..3");
+    if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "no weights");
+    return g->p.u64 ? replay_impl<uint64_t>(g, alg, source, depth, tune, reps, d_label, d_saved, ms, edges, n_active)
+                    : replay_impl<uint32_t>(g, alg, source, depth, tune, reps, d_label, d_saved, ms, edges, n_active);
+}
+
 void etg_free(etg_graph *g) {
     if (!g) return;
     for (int a = 0; a < 4; ++a) {
@@ -529,7 +622,7 @@ void etg_free(etg_graph *g) {
 }
 
 size_t etg_host_scratch_bytes(uint64_t n, uint64_t m, int has_weights, const etg_options *opt) {
-    const Params p = derive(opt);
+    const Params p = derive(opt, env_tune());
     size_t o = 0;
     o = align_up(o + (p.u64 ? 8 : 4) * (n + 1));
     o = align_up(o + 4 * m);
@@ -543,7 +636,7 @@ etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_off, cons
                         size_t scratch_bytes, void *stream, const etg_options *opt, etg_stats *st) {
     if (!h_off || (m && !h_col) || !h_labels || !d_scratch) return fail(ETG_EINVAL, "NULL argument");
     if (alg < 0 || alg > 3) return fail(ETG_EINVAL, "alg must be 0..3");
-    const Params p = derive(opt);
+    const Params p = derive(opt, env_tune());
     const bool has_w = (alg == ALG_SSSP || alg == ALG_SSWP);
     if (has_w && !h_w) return fail(ETG_ENOWEIGHTS, "weights required");
     if (scratch_bytes < etg_host_scratch_bytes(n, m, has_w, opt)) return fail(ETG_ENOMEM, "scratch too small");

@@ -1,32 +1,35 @@
 // etg_kernels.cuh -- sm_100a kernels of the EtaGraph hot path.
 //
-// Per iteration (Proc. 1 while-loop body), three kernels run on
-// the handle's stream with every size kept on the device (no host readback):
+// The active set (Def. 1) of the next iteration is recorded as a bitmap
+// Q of n bits: a relaxation that improves label[u] sets bit u (L136: "the
+// updated vertices are added to the new active set").  Per iteration
+// (Proc. 1 while-loop body) two kernels run on the handle's
+// stream, every size kept on the device:
 //
-//   udc_scan_kernel   step A2 (Def. 3; Sec. IV-A).  Reads the
-//                     raw active set R (vertices activated last iteration), and
-//                     for each v gathers off[v], off[v+1] once: degree-0 vertices
-//                     are dropped ("naturally filter active vertices with
-//                     outdegree equals to 0", L142); the others get
-//                     c = ceil(deg/K) shadow vertices.  A single-pass chained
-//                     (decoupled look-back) scan over the pair (kept, c) writes
-//                     the compacted active set F with, per entry, the start
-//                     offset B, the degree D, the exclusive shadow prefix S,
-//                     and tile_first[t] = the
-//                     entry owning shadow t*TS.  These arrays replace the
-//                     paper's 12-byte 3-tuples (L138): a shadow is recomputed
-//                     from (S, B, D) in O(1) once its entry is known.
 //   expand_kernel     steps A2-A5.  A persistent CTA takes tiles of TS
-//                     consecutive shadows: it loads the tile's window of
-//                     (S, B, D, F) (coalesced), maps each shadow to its slice
-//                     by a binary search in shared memory, stages the tile's
-//                     neighbour segments (<= TS*K words -- the bound UDC gives,
-//                     L199) in shared memory with cp.async (SMP, Sec. V-B
-//                     L197-209), then relaxes every staged edge, one thread per
-//                     edge and kR edges in flight per thread: plain-load
-//                     pre-filter, atomicMin/Max (Proc. 1 L207, reading R-4),
-//                     and a warp-aggregated append of the winners to R (L217).
-//   advance_kernel    step A6: iteration bookkeeping; sets the CUDA-graph
+//                     consecutive shadow vertices: it loads the tile's window
+//                     of the compacted active set (S, B, D, F; coalesced), maps
+//                     each shadow to its slice of at most K out-edges (Def. 3,
+//                     reading R-2) by a binary search in shared memory, stages
+//                     the tile's neighbour segments (<= TS*K words -- the bound
+//                     UDC gives, L199) in shared memory with cp.async (SMP,
+//                     Sec. V-B), then relaxes every staged edge, one
+//                     thread per edge with kR edges in flight: a plain-load
+//                     pre-filter, then a fire-and-forget red.min/red.max (BFS:
+//                     a plain store -- all writers of a level write the same
+//                     depth) and red.or of bit u into Q (Proc. 1 L207, readings
+//                     R-4, R-5).  No thread waits on an atomic's return value.
+//   udc_scan_kernel   steps A5-A6 and the UDC of the next iteration (Def. 3;
+//                     Sec. IV-A).  Reads and clears Q; every set bit v
+//                     gets off[v], off[v+1]; degree-0 vertices are dropped
+//                     ("naturally filter active vertices with outdegree equals
+//                     to 0", L142), the others get c = ceil(deg/K) shadows.  A
+//                     single-pass chained (decoupled look-back) scan over the
+//                     pair (kept, c) writes the compacted active set F with its
+//                     start offsets B, degrees D, exclusive shadow prefix S,
+//                     and tile_first[t] = the entry owning shadow t*TS.  These
+//                     replace the paper's 12-byte 3-tuples (L138).  The last
+//                     scan tile publishes the sizes and sets the CUDA-graph
 //                     conditional ("while actSet.isNotEmpty()", L207).
 #pragma once
 #include <cuda_runtime.h>
@@ -38,26 +41,31 @@ constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr uint32_t kCap = 0xFFFFFFFEu;
 constexpr int kBlock = 256;                 // threads per CTA (8 warps)
 constexpr int kWarps = kBlock / 32;
-constexpr int kScanItems = 8;               // active-set entries per thread in the scan
-constexpr int kScanTile = kBlock * kScanItems;
+constexpr int kScanWords = 4;               // bitmap words per thread in the scan (one uint4)
+constexpr int kScanTile = kBlock * kScanWords;   // words per scan tile (32768 vertices)
 constexpr uint32_t kFull = 0xFFFFFFFFu;
-constexpr int kR = 8;                       // edges in flight per thread in the relax loop
-constexpr uint32_t kQCap = 256;             // per-warp append queue (>= 32 * kR)
+#ifndef ETG_KR
+#define ETG_KR 8
+#endif
+#ifndef ETG_MINB
+#define ETG_MINB 1
+#endif
+constexpr int kR = ETG_KR;                  // edges (chunks) in flight per thread in the relax loop
 
 enum Alg : int { ALG_BFS = 0, ALG_SSSP = 1, ALG_CC = 2, ALG_SSWP = 3 };
 
 // Device-resident control block (one per handle).
 struct Ctl {
-    uint32_t iter;        // iteration index within the current call
-    uint32_t epoch;       // monotone over the handle's life: scan tags and stamps
-    uint32_t count[2];    // raw active-set sizes; count[iter & 1] is the current one
-    uint32_t nF;          // compacted active-set size (entries with out-degree > 0)
-    uint32_t nshadow;     // shadow vertices in the current iteration
-    uint32_t ntiles;      // expand tiles in the current iteration
+    uint32_t depth;       // index of the current active set (BFS: its depth)
+    uint32_t epoch;       // monotone over the handle's life: chained-scan tags
+    uint32_t nF;          // compacted active-set size (vertices with out-degree > 0)
+    uint32_t nshadow;     // shadow vertices of the current active set
+    uint32_t ntiles;      // expand tiles of the current active set
     uint32_t scan_ctr;    // dynamic tile counter of the chained scan
-    uint32_t iterations;  // non-empty iterations of the current call
+    uint32_t tile_ctr;    // dynamic tile counter of the expand
+    uint32_t iterations;  // non-empty active sets expanded in the current call
     uint32_t error;       // ETG_VALIDATE result
-    unsigned long long activations;
+    unsigned long long activations;   // set bits consumed by the scans
     unsigned long long shadows;
     unsigned long long edges;
     unsigned long long frontier;
@@ -73,28 +81,33 @@ struct Dev {
     const OffT *off;
     const uint32_t *col;
     const uint32_t *w;
-    uint32_t *R;                // raw active set (appended by expand, read by scan)
-    uint32_t *F;                // compacted active set (vertex ids)
+    uint32_t *Q;                // next-active-set bitmap (nwords words, zero between uses)
+    uint32_t *F;                // compacted active set (vertex ids, ascending)
     OffT *B;                    // off[F[k]]
     uint32_t *D;                // out-degree of F[k] (> 0)
     uint32_t *S;                // exclusive prefix of shadow counts (nF + 1 entries)
     uint32_t *tile_first;       // entry owning shadow t*ts
-    uint32_t *stamp;            // per-vertex iteration stamp (SSSP/CC/SSWP de-dup)
     uint32_t *st_flag;          // chained scan: per scan tile (epoch << 2 | flag)
     unsigned long long *st_agg; //   aggregate  (entries << 32 | shadows)
     unsigned long long *st_inc; //   inclusive prefix, same packing
     Ctl *ctl;
     uint32_t n;
+    uint32_t nwords;            // bitmap words, a multiple of kScanWords
     uint32_t K;                 // degree limit (Def. 3); unused with NO_UDC
     uint32_t ts;                // shadows per expand tile (<= kBlock, power of 2)
     uint32_t ts_log2;
     uint32_t tune;              // experiment switches (ETG_TUNE env var at load); 0 = default
 };
 
-// tune bits
 constexpr uint32_t kTuneFilterL1 = 1u;    // pre-filter label loads cached in L1
-constexpr uint32_t kTuneMatchAny = 2u;    // suppress same-vertex atomics within a warp
-constexpr uint32_t kTuneBfsStore = 4u;    // EXPERIMENT ONLY: BFS plain store, duplicates kept
+// replay-only experiment switches (etg_debug_expand_replay; results not kept)
+constexpr uint32_t kTuneNoGather = 16u;   // skip the label gather and the commit
+constexpr uint32_t kTuneNoCommit = 32u;   // gather labels but never commit (counts passes)
+constexpr uint32_t kTuneBitOnly = 64u;    // commit = red.or of the bitmap only
+constexpr uint32_t kTuneHashU = 128u;     // targets from a hash of x (no column loads)
+constexpr uint32_t kTuneNoOwner = 256u;   // column index = tile base + x (no owner logic)
+constexpr uint32_t kTuneNoPrefetch = 512u; // no L2 prefetch of the next tile's segments
+constexpr uint32_t kTuneStatic = 1024u;    // static round-robin tile schedule
 
 // ------------------------------------------------------------------------- //
 // small device helpers
@@ -103,11 +116,9 @@ __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
 
 __device__ __forceinline__ uint32_t ld_cg(const uint32_t *p) { return __ldcg(p); }
 
-// Pre-filter load of a label (reading R-4): cached in L1, so a hub's label is
-// fetched once per SM instead of once per in-edge.  Labels move monotonically
-// (down for BFS/SSSP/CC, up for SSWP), so a stale L1 copy can only make the
-// filter pass an edge the atomic then rejects -- never drop an improvement.
-__device__ __forceinline__ uint32_t ld_filter(const uint32_t *p) {
+// L1-cached label load (experiment switch kTuneFilterL1).  Labels move
+// monotonically, so a stale copy can only let the filter pass an edge.
+__device__ __forceinline__ uint32_t ld_ca(const uint32_t *p) {
     uint32_t v;
     asm volatile("ld.global.ca.u32 %0, [%1];" : "=r"(v) : "l"(p));
     return v;
@@ -123,6 +134,52 @@ __device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned lon
     unsigned long long v;
     asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
+}
+
+// L2 residency policies.  The per-vertex arrays (labels, the bitmap) are
+// small and hit randomly: keep them (evict_last).  The edge arrays (col, w)
+// are streamed once per iteration and larger than L2: evict them first, so
+// they do not push the labels out to HBM (where every random 4-byte access
+// would cost a DRAM burst).
+__device__ __forceinline__ uint64_t policy_keep() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t policy_stream() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+// streamed read-only edge data: no L1 allocation, evict-first in L2
+__device__ __forceinline__ uint32_t ld_stream(const uint32_t *p, uint64_t pol) {
+    uint32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+
+// label gather for the pre-filter: L2 only, keep resident
+__device__ __forceinline__ uint32_t ld_label(const uint32_t *p, uint64_t pol) {
+    uint32_t v;
+    asm volatile("ld.global.cg.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+
+// fire-and-forget reductions (no return value: the thread never waits on them)
+__device__ __forceinline__ void red_min(uint32_t *p, uint32_t v, uint64_t pol) {
+    asm volatile("red.relaxed.gpu.global.L2::cache_hint.min.u32 [%0], %1, %2;" :: "l"(p), "r"(v), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void red_max(uint32_t *p, uint32_t v, uint64_t pol) {
+    asm volatile("red.relaxed.gpu.global.L2::cache_hint.max.u32 [%0], %1, %2;" :: "l"(p), "r"(v), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void red_or(uint32_t *p, uint32_t v, uint64_t pol) {
+    asm volatile("red.relaxed.gpu.global.L2::cache_hint.or.b32 [%0], %1, %2;" :: "l"(p), "r"(v), "l"(pol) : "memory");
+}
+
+// bulk L2 prefetch (TMA unit; address and size multiples of 16)
+__device__ __forceinline__ void prefetch_l2(const void *p, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(p), "r"(bytes) : "memory");
 }
 
 __device__ __forceinline__ void cp_async4(void *smem, const void *gmem) {
@@ -142,6 +199,12 @@ __device__ __forceinline__ T warp_incl_scan(T x) {
         T y = __shfl_up_sync(kFull, x, d);
         if (lane_id() >= (uint32_t)d) x += y;
     }
+    return x;
+}
+
+__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long x) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(kFull, x, o);
     return x;
 }
 
@@ -178,10 +241,8 @@ __device__ __forceinline__ uint32_t udc_count(D deg, uint32_t K) {
 // "Init actSet", L207)
 // ------------------------------------------------------------------------- //
 __global__ void ctl_begin_kernel(Ctl *ctl, uint32_t *label, uint32_t source) {
-    ctl->iter = 0;
+    ctl->depth = kInf;            // the first scan makes it 0
     ctl->epoch += 1;
-    ctl->count[0] = 0;
-    ctl->count[1] = 0;
     ctl->nF = 0;
     ctl->nshadow = 0;
     ctl->ntiles = 0;
@@ -195,94 +256,97 @@ __global__ void ctl_begin_kernel(Ctl *ctl, uint32_t *label, uint32_t source) {
     ctl->source = source;
 }
 
-// BFS/SSSP: label = INF, label[s] = 0, R = {s}.  SSWP: label = 0, label[s] =
-// INF.  CC: label[v] = v, R = all vertices (the scan drops degree-0 ones).
+// BFS/SSSP: label = INF, label[s] = 0, Q = {s}.  SSWP: label = 0, label[s] =
+// INF, Q = {s}.  CC: label[v] = v, Q = all vertices (the scan drops degree-0
+// ones).  Q is all-zero on entry (every scan clears what it reads).
 template <class OffT, int ALG>
 __global__ __launch_bounds__(kBlock) void init_kernel(Dev<OffT> d, uint32_t *label, uint32_t source) {
     const uint32_t n = d.n;
     const uint32_t stride = gridDim.x * kBlock;
     for (uint32_t v = blockIdx.x * kBlock + threadIdx.x; v < n; v += stride) {
         uint32_t lab;
-        if (ALG == ALG_CC) {
-            lab = v;
-            d.R[v] = v;
-        } else if (ALG == ALG_SSWP) {
-            lab = (v == source) ? kInf : 0u;
-        } else {
-            lab = (v == source) ? 0u : kInf;
-        }
+        if (ALG == ALG_CC) lab = v;
+        else if (ALG == ALG_SSWP) lab = (v == source) ? kInf : 0u;
+        else lab = (v == source) ? 0u : kInf;
         label[v] = lab;
     }
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        if (ALG == ALG_CC) {
-            d.ctl->count[0] = n;
-        } else {
-            d.R[0] = source;
-            d.ctl->count[0] = 1;
+    if (ALG == ALG_CC) {
+        for (uint32_t k = blockIdx.x * kBlock + threadIdx.x; k < d.nwords; k += stride) {
+            const uint32_t lo = k * 32;
+            d.Q[k] = lo >= n ? 0u : (n - lo >= 32 ? kFull : ((1u << (n - lo)) - 1u));
         }
+    } else if (blockIdx.x == 0 && threadIdx.x == 0) {
+        d.Q[source >> 5] = 1u << (source & 31);
     }
 }
 
 // ------------------------------------------------------------------------- //
-// A2: UDC count + compaction + chained exclusive scan (+ tile_first).
+// A5/A6 + A2 of the next iteration: bitmap -> compacted active set + UDC scan.
 // Persistent CTAs take scan tiles in order from a counter, so the look-back
 // always makes progress.  Values are packed (kept entries << 32 | shadows);
 // neither half can carry into the other (entries <= n < 2^32, shadows < 2^32
-// checked at load time).  The look-back is warp-parallel: warp 0 inspects 32
-// predecessors per step.
+// checked at load time).  The look-back is warp-parallel (32 predecessors per
+// step).  Each thread owns kScanWords consecutive bitmap words.
 // ------------------------------------------------------------------------- //
-__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long x) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(kFull, x, o);
-    return x;
+template <class OffT, bool UDC>
+__device__ __forceinline__ void scan_vertex(const Dev<OffT> &d, uint32_t v, OffT &ob, uint32_t &deg,
+                                            uint32_t &c) {
+    ob = d.off[v];
+    deg = (uint32_t)(d.off[v + 1] - ob);
+    c = udc_count<UDC>(deg, d.K);
 }
 
-template <class OffT, bool UDC>
-__global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d) {
+template <class OffT, bool UDC, bool BFSLAB>
+__global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraphConditionalHandle cond,
+                                                          int use_cond) {
     typedef unsigned long long u64;
     __shared__ uint32_t s_tile;
     __shared__ u64 s_prefix;
     __shared__ u64 s_wsum[kWarps];
     Ctl *ctl = d.ctl;
-    const uint32_t cur = ctl->iter & 1;
-    const uint32_t nR = ctl->count[cur];
     const uint32_t epoch = ctl->epoch & 0x3FFFFFFFu;
-    const uint32_t nscan = (nR + kScanTile - 1) / kScanTile;
+    const uint32_t nscan = (d.nwords + kScanTile - 1) / kScanTile;
     const uint32_t ts = d.ts, tsl = d.ts_log2;
     const uint32_t lane = lane_id();
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        ctl->count[cur ^ 1] = 0;              // the next raw active set starts empty (L140)
-        if (nR == 0) {
-            ctl->nF = 0;
-            ctl->nshadow = 0;
-            ctl->ntiles = 0;
-            d.S[0] = 0;
-        }
-    }
+    uint32_t *label = ctl->label;
+    const uint32_t new_depth = ctl->depth + 1;      // BFS depth of the vertices in Q
     for (;;) {
         if (threadIdx.x == 0) s_tile = atomicAdd(&ctl->scan_ctr, 1u);
         __syncthreads();
         const uint32_t tile = s_tile;
         if (tile >= nscan) break;
-        const uint32_t base = tile * kScanTile + threadIdx.x * kScanItems;
-        uint32_t v[kScanItems], c[kScanItems];
-        OffT ob[kScanItems], deg[kScanItems];
-        u64 tsum = 0;
-#pragma unroll
-        for (int k = 0; k < kScanItems; ++k) v[k] = (base + k < nR) ? d.R[base + k] : kInf;
-#pragma unroll
-        for (int k = 0; k < kScanItems; ++k) {
-            ob[k] = 0;
-            deg[k] = 0;
-            if (v[k] != kInf) {
-                ob[k] = d.off[v[k]];
-                deg[k] = d.off[v[k] + 1] - ob[k];
-            }
+        const uint32_t wbase = tile * kScanTile + threadIdx.x * kScanWords;
+        uint32_t wd[kScanWords] = {0u, 0u, 0u, 0u};
+        if (wbase < d.nwords) {
+            uint4 q = *reinterpret_cast<const uint4 *>(&d.Q[wbase]);
+            wd[0] = q.x; wd[1] = q.y; wd[2] = q.z; wd[3] = q.w;
+            if (q.x | q.y | q.z | q.w) *reinterpret_cast<uint4 *>(&d.Q[wbase]) = make_uint4(0u, 0u, 0u, 0u);
         }
+        // pass 1: (kept, shadows) of this thread's set bits; 4 gathers in flight
+        u64 tsum = 0;
+        uint32_t nbits = 0;
 #pragma unroll
-        for (int k = 0; k < kScanItems; ++k) {
-            c[k] = udc_count<UDC>(deg[k], d.K);
-            tsum += ((u64)(c[k] > 0) << 32) | c[k];
+        for (int k = 0; k < kScanWords; ++k) {
+            uint32_t w = wd[k];
+            nbits += __popc(w);
+            while (w) {
+                uint32_t vv[4], cc[4], dg[4];
+                OffT ob[4];
+#pragma unroll
+                for (int r = 0; r < 4; ++r) {
+                    vv[r] = kInf;
+                    if (w) {
+                        vv[r] = (wbase + k) * 32 + (__ffs(w) - 1);
+                        w &= w - 1;
+                    }
+                }
+#pragma unroll
+                for (int r = 0; r < 4; ++r)
+                    if (vv[r] != kInf) scan_vertex<OffT, UDC>(d, vv[r], ob[r], dg[r], cc[r]);
+#pragma unroll
+                for (int r = 0; r < 4; ++r)
+                    if (vv[r] != kInf) tsum += ((u64)(cc[r] > 0) << 32) | cc[r];
+            }
         }
         u64 btotal;
         const u64 tprefix = block_excl_scan<u64>(tsum, s_wsum, btotal);
@@ -303,7 +367,7 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d) {
                 int p = (int)tile - 1;                  // nearest predecessor in lane 0
                 for (;;) {
                     const int q = p - (int)lane;
-                    uint32_t f = (epoch << 2) | 1u;     // q < 0: beyond tile 0, never used
+                    uint32_t f = (epoch << 2) | 1u;     // q < 0: beyond tile 0, never needed
                     if (q >= 0) f = ld_volatile_u32(&d.st_flag[q]);
                     const bool valid = (f >> 2) == epoch && (f & 3u) != 0;
                     const uint32_t incl = __ballot_sync(kFull, valid && (f & 3u) == 2u && q >= 0);
@@ -328,21 +392,35 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d) {
             if (lane == 0) s_prefix = excl;
         }
         __syncthreads();
+        // pass 2: write the compacted entries (the gathers hit L1 now)
         u64 run = s_prefix + tprefix;
 #pragma unroll
-        for (int k = 0; k < kScanItems; ++k) {
-            if (c[k]) {
-                const uint32_t pos = (uint32_t)(run >> 32);
-                const uint32_t sh = (uint32_t)run;
-                d.F[pos] = v[k];
-                d.B[pos] = ob[k];
-                d.D[pos] = (uint32_t)deg[k];
-                d.S[pos] = sh;
-                // tiles whose first shadow t*ts lies in [sh, sh + c)
-                for (uint32_t t = (sh + ts - 1) >> tsl; (t << tsl) < sh + c[k]; ++t) d.tile_first[t] = pos;
+        for (int k = 0; k < kScanWords; ++k) {
+            uint32_t w = wd[k];
+            while (w) {
+                const uint32_t v = (wbase + k) * 32 + (__ffs(w) - 1);
+                w &= w - 1;
+                if (BFSLAB) label[v] = new_depth;          // BFS: depth written once, on compaction
+                OffT ob;
+                uint32_t dg, c;
+                scan_vertex<OffT, UDC>(d, v, ob, dg, c);
+                if (c) {
+                    const uint32_t pos = (uint32_t)(run >> 32);
+                    const uint32_t sh = (uint32_t)run;
+                    d.F[pos] = v;
+                    d.B[pos] = ob;
+                    d.D[pos] = dg;
+                    d.S[pos] = sh;
+                    // tiles whose first shadow t*ts lies in [sh, sh + c)
+                    for (uint32_t t = (sh + ts - 1) >> tsl; (t << tsl) < sh + c; ++t) d.tile_first[t] = pos;
+                    run += ((u64)1 << 32) | c;
+                }
             }
-            run += ((u64)(c[k] > 0) << 32) | c[k];
         }
+        // activations: one atomic per warp
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) nbits += __shfl_xor_sync(kFull, nbits, o);
+        if (lane == 0 && nbits) atomicAdd(&ctl->activations, (u64)nbits);
         if (tile == nscan - 1 && threadIdx.x == 0) {
             const u64 total = s_prefix + btotal;
             const uint32_t nF = (uint32_t)(total >> 32), N = (uint32_t)total;
@@ -350,6 +428,9 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d) {
             ctl->nF = nF;
             ctl->nshadow = N;
             ctl->ntiles = (N + ts - 1) >> tsl;
+            ctl->tile_ctr = 0;
+            ctl->depth += 1;
+            if (use_cond) cudaGraphSetConditional(cond, nF > 0 ? 1u : 0u);
         }
         __syncthreads();
     }
@@ -407,20 +488,8 @@ __device__ __forceinline__ uint32_t map_shadow(const Dev<OffT> &d, uint32_t i, u
 
 // ------------------------------------------------------------------------- //
 // A4: relaxation (Proc. 1 L207 "if label[v'] > label[v] + 1 then label[v'] =
-// label[v] + 1"), split in three so a thread keeps kR independent edges in
-// flight: candidate -> plain-load pre-filter -> atomic (R-4).  BFS passes the
-// candidate level + 1 as `lab`.
+// label[v] + 1").  BFS passes the candidate level + 1 as `lab`.
 // ------------------------------------------------------------------------- //
-// Copy a warp's queue of qn activated vertices to the raw active set R.
-__device__ __forceinline__ void warp_flush(const uint32_t *wq, uint32_t qn, uint32_t *R,
-                                           uint32_t *cnt) {
-    uint32_t base = 0;
-    if (lane_id() == 0) base = atomicAdd(cnt, qn);
-    base = __shfl_sync(kFull, base, 0);
-    for (uint32_t k = lane_id(); k < qn; k += 32) R[base + k] = wq[k];
-    __syncwarp();
-}
-
 template <int ALG>
 __device__ __forceinline__ uint32_t candidate(uint32_t lab, uint32_t w) {
     if (ALG == ALG_SSSP) {
@@ -438,11 +507,18 @@ __device__ __forceinline__ bool improves(uint32_t cand, uint32_t cur) {
     return cand < cur;
 }
 
-// true iff this thread's atomic lowered (raised, SSWP) the label
+// Commit an improving relaxation.  The plain load saw label[u] worse than
+// cand, so after this label[u] is strictly better than its value at some
+// moment of this iteration: u changed and is active next iteration, whichever
+// thread's value wins (reading R-5: the bitmap de-duplicates).  BFS only sets
+// the bit: every discoverer of u in this iteration would write the same depth,
+// and the scan that compacts u writes it once.
 template <int ALG>
-__device__ __forceinline__ bool atomic_improve(uint32_t *p, uint32_t cand) {
-    if (ALG == ALG_SSWP) return atomicMax(p, cand) < cand;
-    return atomicMin(p, cand) > cand;
+__device__ __forceinline__ void commit(uint32_t *label, uint32_t *Q, uint32_t u, uint32_t cand,
+                                       uint64_t pol) {
+    if (ALG == ALG_SSWP) red_max(&label[u], cand, pol);
+    else if (ALG != ALG_BFS) red_min(&label[u], cand, pol);
+    red_or(&Q[u >> 5], 1u << (u & 31), pol);
 }
 
 // ------------------------------------------------------------------------- //
@@ -468,20 +544,22 @@ __global__ __launch_bounds__(kBlock) void expand_kernel(Dev<OffT> d, uint32_t ca
     uint8_t *sidx = SMP ? reinterpret_cast<uint8_t *>(kW ? (w_s + cap_e) : w_s) : dyn_smem;
 
     Ctl *ctl = d.ctl;
-    const uint32_t it = ctl->iter, nxt = (it & 1) ^ 1;
     const uint32_t nF = ctl->nF, N = ctl->nshadow, ntiles = ctl->ntiles;
-    const uint32_t tag = ctl->epoch;
+    const uint32_t level = ctl->depth + 1;
     uint32_t *label = ctl->label;
-    uint32_t *Rn = d.R;
-    uint32_t *cnt_n = &ctl->count[nxt];
-    const uint32_t level = it + 1;
-    const uint32_t lane = lane_id();
+    uint32_t *Q = d.Q;
     const uint32_t tid = threadIdx.x;
+    const bool l1 = (d.tune & kTuneFilterL1) != 0;
+    const uint64_t keep = policy_keep();
     unsigned long long my_edges = 0;
-    uint32_t my_acts = 0;
-    __shared__ uint32_t s_queue[kWarps][kQCap];    // per-warp queue of activated vertices
-    uint32_t *wq = s_queue[tid >> 5];
-    uint32_t qn = 0;                                // warp-uniform queue length
+    if (blockIdx.x == 0 && tid == 0) {
+        // bookkeeping for the scan that follows this kernel (stream-ordered)
+        ctl->scan_ctr = 0;
+        ctl->epoch += 1;
+        if (nF) ctl->iterations += 1;
+        ctl->frontier += nF;
+        ctl->shadows += N;
+    }
 
     for (uint32_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
         const uint32_t W = load_window<OffT, kLab>(d, t, nF, win);
@@ -522,8 +600,8 @@ __global__ __launch_bounds__(kBlock) void expand_kernel(Dev<OffT> d, uint32_t ca
             cp_async_wait_all();
             __syncthreads();
         }
-        // A4 + A5 in batches of kR edges per thread: all loads of a batch are
-        // issued before any is consumed (memory-level parallelism).
+        // A4 + A5 in batches of kR edges per thread: the batch's label loads
+        // are all issued before any is consumed; commits never wait.
         for (uint32_t x0 = 0; x0 < E; x0 += kBlock * kR) {
             uint32_t u[kR], c[kR], cur[kR];
             bool act[kR];
@@ -558,93 +636,237 @@ __global__ __launch_bounds__(kBlock) void expand_kernel(Dev<OffT> d, uint32_t ca
             }
 #pragma unroll
             for (int r = 0; r < kR; ++r)
-                cur[r] = act[r] ? ((d.tune & kTuneFilterL1) ? ld_filter(&label[u[r]]) : ld_cg(&label[u[r]])) : 0u;
+                cur[r] = act[r] ? (l1 ? ld_ca(&label[u[r]]) : ld_cg(&label[u[r]])) : 0u;
 #pragma unroll
-            for (int r = 0; r < kR; ++r) act[r] = act[r] && improves<ALG>(c[r], cur[r]);
-            if (d.tune & kTuneMatchAny) {
-#pragma unroll
-                for (int r = 0; r < kR; ++r) {
-                    const uint32_t peers = __match_any_sync(kFull, act[r] ? u[r] : kInf);
-                    // among lanes proposing the same vertex keep the best candidate
-                    // (BFS: all equal, so the lowest lane)
-                    uint32_t best = act[r] ? c[r] : (ALG == ALG_SSWP ? 0u : kInf);
-                    for (uint32_t m = peers; m; m &= m - 1) {
-                        const uint32_t o = __shfl_sync(peers, best, __ffs(m) - 1);
-                        (void)o;
-                    }
-                    if (act[r] && (peers & ((1u << lane) - 1)) && ALG == ALG_BFS) act[r] = false;
-                }
-            }
-            if (ALG == ALG_BFS && (d.tune & kTuneBfsStore)) {
-#pragma unroll
-                for (int r = 0; r < kR; ++r)
-                    if (act[r]) label[u[r]] = c[r];
-            } else {
-#pragma unroll
-                for (int r = 0; r < kR; ++r)
-                    if (act[r]) act[r] = atomic_improve<ALG>(&label[u[r]], c[r]);
-            }
-            if (ALG != ALG_BFS) {                              // once per iteration (R-5)
-#pragma unroll
-                for (int r = 0; r < kR; ++r)
-                    if (act[r]) act[r] = atomicExch(&d.stamp[u[r]], tag) != tag;
-            }
-            // A5: append the winners to the warp's shared-memory queue; the
-            // queue is flushed to R with ONE atomicAdd per kQCap entries
-            // (L217's atomic append, aggregated: a single global counter would
-            // otherwise serialise every warp of the grid).
-            uint32_t masks[kR], total = 0;
-#pragma unroll
-            for (int r = 0; r < kR; ++r) {
-                masks[r] = __ballot_sync(kFull, act[r]);
-                total += __popc(masks[r]);
-            }
-            if (total) {
-                if (qn + total > kQCap) {
-                    warp_flush(wq, qn, Rn, cnt_n);
-                    qn = 0;
-                }
-                uint32_t base = qn;
-                const uint32_t lt = (1u << lane) - 1;
-#pragma unroll
-                for (int r = 0; r < kR; ++r) {
-                    if (act[r]) wq[base + __popc(masks[r] & lt)] = u[r];
-                    base += __popc(masks[r]);
-                }
-                qn += total;
-                my_acts += (lane == 0) ? total : 0u;
-                __syncwarp();
-            }
+            for (int r = 0; r < kR; ++r)
+                if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep);
         }
         my_edges += E;
         __syncthreads();
     }
-    if (qn) warp_flush(wq, qn, Rn, cnt_n);
-    // statistics: one atomic per CTA
-    __shared__ uint32_t s_acts[kWarps];
-    if (lane == 0) s_acts[tid >> 5] = my_acts;
-    __syncthreads();
-    if (tid == 0) {
-        uint32_t a = 0;
-        for (int k = 0; k < kWarps; ++k) a += s_acts[k];
-        if (a) atomicAdd(&ctl->activations, (unsigned long long)a);
-        if (my_edges) atomicAdd(&ctl->edges, my_edges);
-    }
+    if (tid == 0 && my_edges) atomicAdd(&ctl->edges, my_edges);
 }
 
 // ------------------------------------------------------------------------- //
-// A6: iteration control (Proc. 1 "while actSet.isNotEmpty()", L207; reset of
-// the consumed active set, L140).
+// Warp-centric expand (the default).  One warp owns a tile of 32 consecutive
+// shadow vertices (ts = 32) and processes it with registers and warp
+// intrinsics only -- no shared memory, no block barrier -- so the random label
+// gathers are the only traffic in the SM's memory pipe.
+//
+// warp_map: lane i gets shadow t*32 + i.  The tile's entries j0 .. j0+31
+// (j0 = tile_first[t]) are loaded one per lane; entry j > j0 starts a shadow
+// inside the tile at position p_j = S[j] - 32t, so OR-reducing 1 << p_j gives
+// the mask of entry starts, and the entry owning position i is j0 plus the
+// number of starts at positions <= i (entry j0 covers position 0).
 // ------------------------------------------------------------------------- //
-__global__ void advance_kernel(Ctl *ctl, cudaGraphConditionalHandle cond, int use_cond) {
-    const uint32_t cur = ctl->iter & 1;
-    if (ctl->nF > 0) ctl->iterations += 1;
-    ctl->frontier += ctl->nF;
-    ctl->shadows += ctl->nshadow;
-    ctl->iter += 1;
-    ctl->epoch += 1;
-    ctl->scan_ctr = 0;
-    if (use_cond) cudaGraphSetConditional(cond, ctl->count[cur ^ 1] > 0 ? 1u : 0u);
+template <class OffT, bool UDC>
+struct WarpShadow {
+    OffT start;
+    uint32_t len;
+    uint32_t v;
+};
+
+template <class OffT, bool UDC>
+__device__ __forceinline__ WarpShadow<OffT, UDC> warp_map(const Dev<OffT> &d, uint32_t t, uint32_t nF,
+                                                          uint32_t N) {
+    const uint32_t lane = lane_id();
+    const uint32_t j0 = d.tile_first[t];
+    const uint32_t j = j0 + lane;
+    uint32_t Sj = kInf, Dj = 0, Fj = 0;
+    OffT Bj = 0;
+    if (j < nF) {
+        Sj = d.S[j];
+        Bj = d.B[j];
+        Dj = d.D[j];
+        Fj = d.F[j];
+    }
+    const uint32_t base = t << 5;
+    const uint32_t p = Sj - base;                              // wraps to huge if Sj < base
+    const uint32_t startmask = __reduce_or_sync(kFull, (lane > 0 && p < 32u) ? (1u << p) : 0u);
+    const uint32_t jj = __popc(startmask & ((2u << lane) - 1u));
+    const uint32_t sS = __shfl_sync(kFull, Sj, jj);
+    const OffT sB = __shfl_sync(kFull, Bj, jj);
+    const uint32_t sD = __shfl_sync(kFull, Dj, jj);
+    WarpShadow<OffT, UDC> r;
+    r.v = __shfl_sync(kFull, Fj, jj);
+    r.len = 0;
+    r.start = 0;
+    const uint32_t i = base + lane;
+    if (i < N) {
+        if (UDC) {
+            const uint32_t qk = (i - sS) * d.K;              // < deg
+            r.start = sB + (OffT)qk;
+            const uint32_t rem = sD - qk;
+            r.len = rem < d.K ? rem : d.K;
+        } else {
+            r.start = sB;
+            r.len = sD;
+        }
+    }
+    return r;
+}
+
+template <class OffT, int ALG, bool UDC>
+__global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT> d) {
+    constexpr bool kW = (ALG == ALG_SSSP || ALG == ALG_SSWP);
+    Ctl *ctl = d.ctl;
+    const uint32_t nF = ctl->nF, N = ctl->nshadow, ntiles = ctl->ntiles;
+    const uint32_t level = ctl->depth + 1;
+    uint32_t *label = ctl->label;
+    uint32_t *Q = d.Q;
+    const uint32_t lane = lane_id();
+    const uint32_t lt_eq = (2u << lane) - 1u;
+    const bool l1 = (d.tune & kTuneFilterL1) != 0;
+    const uint64_t keep = policy_keep(), stream = policy_stream();
+    unsigned long long my_edges = 0;
+    uint32_t my_passes = 0;                               // replay experiment counter
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        // bookkeeping for the scan that follows this kernel (stream-ordered)
+        ctl->scan_ctr = 0;
+        ctl->epoch += 1;
+        if (nF) ctl->iterations += 1;
+        ctl->frontier += nF;
+        ctl->shadows += N;
+    }
+    // Dynamic schedule: a warp grabs kGrab consecutive tiles at a time, so the
+    // slowest warp ends within one grab of the rest (tiles carry 32..32K edges).
+    // One-tile lookahead: the next tile is mapped, and its neighbour segments
+    // are prefetched into L2 (cp.async.bulk.prefetch), while the current tile is
+    // relaxed, so its column reads hit L2 instead of waiting on HBM.
+    constexpr uint32_t kGrab = 2;
+    uint32_t g_next = 0, g_end = 0;
+    const uint32_t gwarp = blockIdx.x * kWarps + (threadIdx.x >> 5), nwarps = gridDim.x * kWarps;
+    uint32_t s_next = gwarp;
+    auto next_tile = [&]() -> uint32_t {
+        if (d.tune & kTuneStatic) {                       // static round-robin (experiment)
+            const uint32_t r = s_next;
+            s_next += nwarps;
+            return r < ntiles ? r : ntiles;
+        }
+        if (g_next == g_end) {
+            uint32_t g = 0;
+            if (lane == 0) g = atomicAdd(&ctl->tile_ctr, kGrab);
+            g_next = __shfl_sync(kFull, g, 0);
+            g_end = g_next >= ntiles ? g_next : min(g_next + kGrab, ntiles);
+            if (g_next >= ntiles) return ntiles;
+        }
+        return g_next++;
+    };
+    auto prefetch = [&](const WarpShadow<OffT, UDC> &w) {
+        if (w.len && !(d.tune & kTuneNoPrefetch)) {
+            const uintptr_t lo = reinterpret_cast<uintptr_t>(d.col + w.start) & ~(uintptr_t)15;
+            const uintptr_t hi = (reinterpret_cast<uintptr_t>(d.col + w.start + w.len) + 15) & ~(uintptr_t)15;
+            prefetch_l2(reinterpret_cast<const void *>(lo), (uint32_t)(hi - lo));
+            if (kW) prefetch_l2(reinterpret_cast<const void *>(lo - reinterpret_cast<uintptr_t>(d.col) +
+                                                               reinterpret_cast<uintptr_t>(d.w)),
+                                (uint32_t)(hi - lo));
+        }
+    };
+    uint32_t t = next_tile();
+    if (t >= ntiles) {
+        if (lane == 0 && my_edges) atomicAdd(&ctl->edges, my_edges);
+        return;
+    }
+    WarpShadow<OffT, UDC> sh_next = warp_map<OffT, UDC>(d, t, nF, N);
+    prefetch(sh_next);
+    for (;;) {
+        const WarpShadow<OffT, UDC> sh = sh_next;
+        const uint32_t tn = next_tile();
+        if (tn < ntiles) {
+            sh_next = warp_map<OffT, UDC>(d, tn, nF, N);
+            prefetch(sh_next);
+        }
+        const uint32_t lab = (ALG == ALG_BFS) ? level
+                             : (sh.len ? ld_cg(&label[sh.v]) : 0u);   // fresh source label (R-6)
+        const uint32_t incl = warp_incl_scan(sh.len);
+        const uint32_t o = incl - sh.len;                     // flat offset of this lane's slice
+        const OffT delta = sh.start - (OffT)o;                // col index of element x = delta + x
+        const uint32_t E = __shfl_sync(kFull, incl, 31);
+        my_edges += E;
+        uint32_t owner = 0xFFFFFFFFu;                         // owner of the element before x0
+        // Software pipeline over batches of kR chunks (32 elements each): the
+        // column loads of batch b+1 are issued before the label gathers of
+        // batch b, so a warp always has gathers or column loads in flight.
+        uint32_t un[kR], cn[kR];
+        bool an[kR];
+        auto fetch = [&](uint32_t x0) {
+#pragma unroll
+            for (int r = 0; r < kR; ++r) {
+                const uint32_t cx = x0 + 32u * r;            // chunk start
+                const uint32_t pos = o - cx;                  // this lane's slice start in the chunk
+                uint32_t sm = 0;
+                if (!(d.tune & kTuneNoOwner))
+                    sm = __reduce_or_sync(kFull, (sh.len && pos < 32u) ? (1u << pos) : 0u);
+                const uint32_t own = owner + __popc(sm & lt_eq);
+                owner += __popc(sm);
+                const uint32_t src = own & 31u;
+                const OffT dl = (d.tune & kTuneNoOwner) ? __shfl_sync(kFull, delta, 0) : __shfl_sync(kFull, delta, src);
+                const uint32_t ll = (ALG == ALG_BFS) ? level : __shfl_sync(kFull, lab, src);
+                const uint32_t x = cx + lane;
+                an[r] = x < E;
+                un[r] = 0;
+                cn[r] = ll;
+                if (an[r]) {
+                    const OffT e = dl + (OffT)x;
+                    if (d.tune & kTuneHashU) {
+                        uint32_t h = (uint32_t)e * 0x9E3779B1u;
+                        h ^= h >> 15;
+                        h *= 0x85EBCA77u;
+                        h ^= h >> 13;
+                        un[r] = h % d.n;
+                    } else {
+                        un[r] = ld_stream(&d.col[e], stream);
+                    }
+                    if (kW) cn[r] = candidate<ALG>(ll, ld_stream(&d.w[e], stream));
+                }
+            }
+        };
+        fetch(0);
+        for (uint32_t x0 = 0; x0 < E; x0 += 32u * kR) {
+            uint32_t u[kR], c[kR], cur[kR];
+            bool act[kR];
+#pragma unroll
+            for (int r = 0; r < kR; ++r) {
+                u[r] = un[r];
+                c[r] = cn[r];
+                act[r] = an[r];
+            }
+            if (x0 + 32u * kR < E) fetch(x0 + 32u * kR);      // next batch's column loads
+            if (d.tune & kTuneNoGather) {                     // replay experiment
+                uint32_t x = 0;
+#pragma unroll
+                for (int r = 0; r < kR; ++r) x += act[r] ? u[r] + c[r] : 0u;
+                if (x == 0x9E3779B9u) Q[0] = x;
+                continue;
+            }
+#pragma unroll
+            for (int r = 0; r < kR; ++r)
+                cur[r] = act[r] ? (l1 ? ld_ca(&label[u[r]]) : ld_label(&label[u[r]], keep)) : 0u;
+            if (d.tune & kTuneNoCommit) {                     // replay experiment: count passes
+                uint32_t x = 0;
+#pragma unroll
+                for (int r = 0; r < kR; ++r) x += (act[r] && improves<ALG>(c[r], cur[r])) ? 1u : 0u;
+                my_passes += x;
+                continue;
+            }
+            if (d.tune & kTuneBitOnly) {                      // replay experiment: bitmap only
+#pragma unroll
+                for (int r = 0; r < kR; ++r)
+                    if (act[r] && improves<ALG>(c[r], cur[r])) red_or(&Q[u[r] >> 5], 1u << (u[r] & 31), keep);
+                continue;
+            }
+#pragma unroll
+            for (int r = 0; r < kR; ++r)
+                if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep);
+        }
+        if (tn >= ntiles) break;
+    }
+    // statistics: one atomic per warp
+    if (lane == 0 && my_edges) atomicAdd(&ctl->edges, my_edges);
+    if (d.tune & kTuneNoCommit) {
+        my_passes = __reduce_add_sync(kFull, my_passes);
+        if (lane == 0 && my_passes) atomicAdd(&ctl->reached_v, (unsigned long long)my_passes);
+    }
 }
 
 // ------------------------------------------------------------------------- //
@@ -657,7 +879,7 @@ __global__ __launch_bounds__(kBlock) void udc_dump_kernel(Dev<OffT> d, uint32_t 
     Ctl *ctl = d.ctl;
     const uint32_t nF = ctl->nF, N = ctl->nshadow, ntiles = ctl->ntiles;
     for (uint32_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        const uint32_t W = load_window<OffT, false>(d, t, nF, win);
+        const uint32_t W = load_window<OffT, true>(d, t, nF, win);
         const uint32_t cnt = min(d.ts, N - (t << d.ts_log2));
         __syncthreads();
         if (threadIdx.x < cnt) {
@@ -665,12 +887,18 @@ __global__ __launch_bounds__(kBlock) void udc_dump_kernel(Dev<OffT> d, uint32_t 
             OffT start;
             uint32_t len;
             const uint32_t jj = map_shadow<OffT, UDC>(d, i, W, win, start, len);
-            out_id[i] = d.F[d.tile_first[t] + jj];
+            out_id[i] = win.F[jj];
             out_start[i] = (uint64_t)start;
             out_end[i] = (uint64_t)start + len;
         }
         __syncthreads();
     }
+}
+
+// Mark the vertices of an explicit active set in Q (debug entry etg_udc_slices).
+__global__ void mark_kernel(uint32_t *Q, const uint32_t *act, uint32_t n_act) {
+    for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < n_act; k += gridDim.x * blockDim.x)
+        atomicOr(&Q[act[k] >> 5], 1u << (act[k] & 31));
 }
 
 // ------------------------------------------------------------------------- //
@@ -701,8 +929,10 @@ __global__ __launch_bounds__(kBlock) void validate_kernel(Dev<OffT> d, unsigned 
     const uint64_t gsz = (uint64_t)gridDim.x * kBlock;
     const uint64_t t0 = (uint64_t)blockIdx.x * kBlock + threadIdx.x;
     if (t0 == 0 && (d.off[0] != 0 || (unsigned long long)d.off[d.n] != m)) atomicOr(&d.ctl->error, 1u);
-    for (uint64_t v = t0; v < d.n; v += gsz)
+    for (uint64_t v = t0; v < d.n; v += gsz) {
         if (d.off[v + 1] < d.off[v]) atomicOr(&d.ctl->error, 2u);
+        else if ((unsigned long long)(d.off[v + 1] - d.off[v]) > 0xFFFFFFFFull) atomicOr(&d.ctl->error, 8u);
+    }
     for (uint64_t e = t0; e < m; e += gsz)
         if (d.col[e] >= d.n) atomicOr(&d.ctl->error, 4u);
 }

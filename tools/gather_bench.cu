@@ -54,7 +54,7 @@ void run(const char *name, const uint32_t *idx, uint32_t *lab, uint64_t n_idx, u
            5.0 * n_idx / (ms * 1e-3) / 1e9);
 }
 
-int main() {
+int main(int argc, char **argv) {
     int sms;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
     const uint32_t n = 1u << 22;                 // C2 label array: 16.8 MB
@@ -66,6 +66,15 @@ int main() {
     cudaMemset(lab, 0xFF, (uint64_t)n * 4);
     fill_idx<<<sms * 8, 256>>>(idx, n_idx, n, 1);
     cudaDeviceSynchronize();
+    if (argc > 1) {                 // index stream from a file of uint32 (e.g. the C2 col array)
+        FILE *f = fopen(argv[1], "rb");
+        uint32_t *h = (uint32_t *)malloc(n_idx * 4);
+        size_t got = fread(h, 4, n_idx, f);
+        fclose(f);
+        printf("loaded %zu indices from %s\n", got, argv[1]);
+        cudaMemcpy(idx, h, got * 4, cudaMemcpyHostToDevice);
+        free(h);
+    }
     for (int bps : {4, 8}) {
         run<1, 0>("ld.cg", idx, lab, n_idx, out, sms, bps, 256);
         run<8, 0>("ld.cg", idx, lab, n_idx, out, sms, bps, 256);
