@@ -99,9 +99,10 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
     };
     const uint64_t max_shadows = p.udc ? (m + p.K - 1) / p.K + n : n;   // sum ceil(d/K) <= m/K + |F|
     const uint64_t max_tiles = (max_shadows + 31) / 32 + 2;      // sized for the smallest tile (32)
-    const uint64_t max_scan_tiles = ((n + 31) / 32 + kScanTile - 1) / kScanTile + 2;
+    const uint64_t max_scan_tiles = (n + kScanV - 1) / kScanV + 2;
     const uint64_t words = (n + 31) / 32;
-    L.nwords = (uint32_t)((words + kScanWords - 1) / kScanWords * kScanWords);
+    const uint64_t tile_words = kScanV / 32;
+    L.nwords = (uint32_t)((words + tile_words - 1) / tile_words * tile_words);
     L.Q = take(4ull * L.nwords);
     L.F = take(4 * (n + 1));
     L.B = take((p.u64 ? 8 : 4) * (n + 1));
@@ -550,7 +551,7 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
         return bail(fail(ETG_ECUDA, std::string("load: ") + cudaGetErrorString(e)));
     }
     g->tune = tune;
-    g->grid_scan = g->num_sms * 2;
+    g->grid_scan = g->num_sms * 4;
     g->grid_init = g->num_sms * 8;
     if (flags & ETG_VALIDATE) {
         etg_status s = p.u64 ? validate_impl<uint64_t>(g) : validate_impl<uint32_t>(g);

@@ -41,8 +41,6 @@ constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr uint32_t kCap = 0xFFFFFFFEu;
 constexpr int kBlock = 256;                 // threads per CTA (8 warps)
 constexpr int kWarps = kBlock / 32;
-constexpr int kScanWords = 4;               // bitmap words per thread in the scan (one uint4)
-constexpr int kScanTile = kBlock * kScanWords;   // words per scan tile (32768 vertices)
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 #ifndef ETG_KR
 #define ETG_KR 8
@@ -92,7 +90,7 @@ struct Dev {
     unsigned long long *st_inc; //   inclusive prefix, same packing
     Ctl *ctl;
     uint32_t n;
-    uint32_t nwords;            // bitmap words, a multiple of kScanWords
+    uint32_t nwords;            // bitmap words (padded to whole scan tiles)
     uint32_t K;                 // degree limit (Def. 3); unused with NO_UDC
     uint32_t ts;                // shadows per expand tile (<= kBlock, power of 2)
     uint32_t ts_log2;
@@ -282,18 +280,42 @@ __global__ __launch_bounds__(kBlock) void init_kernel(Dev<OffT> d, uint32_t *lab
 
 // ------------------------------------------------------------------------- //
 // A5/A6 + A2 of the next iteration: bitmap -> compacted active set + UDC scan.
-// Persistent CTAs take scan tiles in order from a counter, so the look-back
-// always makes progress.  Values are packed (kept entries << 32 | shadows);
-// neither half can carry into the other (entries <= n < 2^32, shadows < 2^32
-// checked at load time).  The look-back is warp-parallel (32 predecessors per
-// step).  Each thread owns kScanWords consecutive bitmap words.
+// Scan tile = kScanV vertices; thread tid owns the kVT consecutive vertices
+// v0 = tile*kScanV + tid*kVT .. v0+kVT-1: their kVT bits of Q and, when any is
+// set, the kVT+1 row offsets off[v0 .. v0+kVT] read with vector loads
+// (coalesced across the warp), from which every degree follows -- no per-
+// vertex gather and no second gather in pass 2.  Persistent CTAs take scan
+// tiles in order from a counter, so the look-back always makes progress.
+// Values are packed (kept entries << 32 | shadows); neither half can carry
+// into the other (entries <= n < 2^32, shadows < 2^32 checked at load time).
+// The look-back is warp-parallel (32 predecessors per step).
 // ------------------------------------------------------------------------- //
-template <class OffT, bool UDC>
-__device__ __forceinline__ void scan_vertex(const Dev<OffT> &d, uint32_t v, OffT &ob, uint32_t &deg,
-                                            uint32_t &c) {
-    ob = d.off[v];
-    deg = (uint32_t)(d.off[v + 1] - ob);
-    c = udc_count<UDC>(deg, d.K);
+constexpr int kVT = 32;                          // vertices per thread (one bitmap word)
+constexpr uint32_t kScanV = kBlock * kVT;        // vertices per scan tile (8192 = 256 words)
+
+template <class OffT>
+__device__ __forceinline__ void load_offsets(const OffT *off, uint32_t v0, uint32_t n, OffT (&o)[kVT + 1]) {
+    if (v0 + kVT <= n) {
+        if (sizeof(OffT) == 4) {
+            const uint4 *p = reinterpret_cast<const uint4 *>(off + v0);
+#pragma unroll
+            for (int k = 0; k < kVT / 4; ++k) {
+                const uint4 q = __ldg(p + k);
+                o[4 * k] = (OffT)q.x; o[4 * k + 1] = (OffT)q.y; o[4 * k + 2] = (OffT)q.z; o[4 * k + 3] = (OffT)q.w;
+            }
+        } else {
+            const ulonglong2 *p = reinterpret_cast<const ulonglong2 *>(off + v0);
+#pragma unroll
+            for (int k = 0; k < kVT / 2; ++k) {
+                const ulonglong2 q = __ldg(p + k);
+                o[2 * k] = (OffT)q.x; o[2 * k + 1] = (OffT)q.y;
+            }
+        }
+        o[kVT] = __ldg(off + v0 + kVT);
+    } else {
+#pragma unroll
+        for (int k = 0; k <= kVT; ++k) o[k] = (v0 + k <= n) ? __ldg(off + v0 + k) : (OffT)0;
+    }
 }
 
 template <class OffT, bool UDC, bool BFSLAB>
@@ -305,7 +327,8 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
     __shared__ u64 s_wsum[kWarps];
     Ctl *ctl = d.ctl;
     const uint32_t epoch = ctl->epoch & 0x3FFFFFFFu;
-    const uint32_t nscan = (d.nwords + kScanTile - 1) / kScanTile;
+    const uint32_t n = d.n;
+    const uint32_t nscan = (n + kScanV - 1) / kScanV;
     const uint32_t ts = d.ts, tsl = d.ts_log2;
     const uint32_t lane = lane_id();
     uint32_t *label = ctl->label;
@@ -315,37 +338,20 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
         __syncthreads();
         const uint32_t tile = s_tile;
         if (tile >= nscan) break;
-        const uint32_t wbase = tile * kScanTile + threadIdx.x * kScanWords;
-        uint32_t wd[kScanWords] = {0u, 0u, 0u, 0u};
-        if (wbase < d.nwords) {
-            uint4 q = *reinterpret_cast<const uint4 *>(&d.Q[wbase]);
-            wd[0] = q.x; wd[1] = q.y; wd[2] = q.z; wd[3] = q.w;
-            if (q.x | q.y | q.z | q.w) *reinterpret_cast<uint4 *>(&d.Q[wbase]) = make_uint4(0u, 0u, 0u, 0u);
-        }
-        // pass 1: (kept, shadows) of this thread's set bits; 4 gathers in flight
+        const uint32_t v0 = tile * kScanV + threadIdx.x * kVT;
+        // this thread's bitmap word (read and cleared)
+        const uint32_t bits = v0 < n ? d.Q[v0 >> 5] : 0u;
+        if (bits) d.Q[v0 >> 5] = 0u;
+        OffT o[kVT + 1];
         u64 tsum = 0;
-        uint32_t nbits = 0;
+        if (bits) {
+            load_offsets<OffT>(d.off, v0, n, o);
 #pragma unroll
-        for (int k = 0; k < kScanWords; ++k) {
-            uint32_t w = wd[k];
-            nbits += __popc(w);
-            while (w) {
-                uint32_t vv[4], cc[4], dg[4];
-                OffT ob[4];
-#pragma unroll
-                for (int r = 0; r < 4; ++r) {
-                    vv[r] = kInf;
-                    if (w) {
-                        vv[r] = (wbase + k) * 32 + (__ffs(w) - 1);
-                        w &= w - 1;
-                    }
+            for (int k = 0; k < kVT; ++k) {
+                if (bits & (1u << k)) {
+                    const uint32_t c = udc_count<UDC>((OffT)(o[k + 1] - o[k]), d.K);
+                    tsum += ((u64)(c > 0) << 32) | c;
                 }
-#pragma unroll
-                for (int r = 0; r < 4; ++r)
-                    if (vv[r] != kInf) scan_vertex<OffT, UDC>(d, vv[r], ob[r], dg[r], cc[r]);
-#pragma unroll
-                for (int r = 0; r < 4; ++r)
-                    if (vv[r] != kInf) tsum += ((u64)(cc[r] > 0) << 32) | cc[r];
             }
         }
         u64 btotal;
@@ -392,35 +398,33 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
             if (lane == 0) s_prefix = excl;
         }
         __syncthreads();
-        // pass 2: write the compacted entries (the gathers hit L1 now)
-        u64 run = s_prefix + tprefix;
+        // pass 2: write the compacted entries (offsets still in registers)
+        if (bits) {
+            u64 run = s_prefix + tprefix;
 #pragma unroll
-        for (int k = 0; k < kScanWords; ++k) {
-            uint32_t w = wd[k];
-            while (w) {
-                const uint32_t v = (wbase + k) * 32 + (__ffs(w) - 1);
-                w &= w - 1;
-                if (BFSLAB) label[v] = new_depth;          // BFS: depth written once, on compaction
-                OffT ob;
-                uint32_t dg, c;
-                scan_vertex<OffT, UDC>(d, v, ob, dg, c);
-                if (c) {
-                    const uint32_t pos = (uint32_t)(run >> 32);
-                    const uint32_t sh = (uint32_t)run;
-                    d.F[pos] = v;
-                    d.B[pos] = ob;
-                    d.D[pos] = dg;
-                    d.S[pos] = sh;
-                    // tiles whose first shadow t*ts lies in [sh, sh + c)
-                    for (uint32_t t = (sh + ts - 1) >> tsl; (t << tsl) < sh + c; ++t) d.tile_first[t] = pos;
-                    run += ((u64)1 << 32) | c;
+            for (int k = 0; k < kVT; ++k) {
+                if (bits & (1u << k)) {
+                    const uint32_t v = v0 + k;
+                    if (BFSLAB) label[v] = new_depth;      // BFS: depth written once, on compaction
+                    const uint32_t dg = (uint32_t)(o[k + 1] - o[k]);
+                    const uint32_t c = udc_count<UDC>(dg, d.K);
+                    if (c) {
+                        const uint32_t pos = (uint32_t)(run >> 32);
+                        const uint32_t sh = (uint32_t)run;
+                        d.F[pos] = v;
+                        d.B[pos] = o[k];
+                        d.D[pos] = dg;
+                        d.S[pos] = sh;
+                        // tiles whose first shadow t*ts lies in [sh, sh + c)
+                        for (uint32_t t = (sh + ts - 1) >> tsl; (t << tsl) < sh + c; ++t) d.tile_first[t] = pos;
+                        run += ((u64)1 << 32) | c;
+                    }
                 }
             }
         }
         // activations: one atomic per warp
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) nbits += __shfl_xor_sync(kFull, nbits, o);
-        if (lane == 0 && nbits) atomicAdd(&ctl->activations, (u64)nbits);
+        const uint32_t nbits = __reduce_add_sync(kFull, (uint32_t)__popc(bits));
+        if (lane == 0 && nbits) atomicAdd(&ctl->activations, (u64)nbits);   // result unused: RED
         if (tile == nscan - 1 && threadIdx.x == 0) {
             const u64 total = s_prefix + btotal;
             const uint32_t nF = (uint32_t)(total >> 32), N = (uint32_t)total;
