@@ -170,9 +170,10 @@ def ncu_traffic(config):
     try:
         with open(path) as f:
             d = json.load(f)
-        return d.get(config, {}).get("dram_bytes_per_launch")
+        c = d.get(config, {})
+        return c.get("dram_bytes_per_launch"), c.get("algorithmic_bytes_of_captured_launch")
     except (OSError, ValueError):
-        return None
+        return None, None
 
 
 # --------------------------------------------------------------------------- #
@@ -414,9 +415,12 @@ def run_ours(args):
                 d["edges_processed"] += st.edges_processed
         peak, peak_src = measured_peak()
         achieved = bytes_tot / (exp_ms * 1e-3) / 1e9
-        traffic = ncu_traffic(args.config)
+        traffic, traffic_alg = ncu_traffic(args.config)
         roof = {"bound": "hbm", "kernel": "expand_kernel", "achieved": achieved, "peak": peak,
                 "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                "traffic_note": ("dram read+write bytes of one ncu --set full capture of the largest BFS "
+                                 "expand launch (profiles/expand_ncu_summary.json); algorithmic bytes of "
+                                 f"that launch: {traffic_alg}") if traffic else None,
                 "peak_source": peak_src,
                 "algorithmic_bytes_per_launch": bytes_tot / max(1, launches_p),
                 "avg_launch_ms": exp_ms / max(1, launches_p),
@@ -472,7 +476,7 @@ def run_ours(args):
     # ---- CPU oracle baseline (rank 0, N = 1 only) ----
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        e, secs, sample = oracle_leg(args.config, algs, args.sources, 4242, budget_s=20.0, g=g, gs=gs)
+        e, secs, sample = oracle_leg(args.config, algs, args.sources, 4242, budget_s=12.0, g=g, gs=gs)
         cpu = {"value": e / secs / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
                "sample": f"{sample} on {args.config} (single-threaded C oracle, {os.cpu_count()} host cores present)"}
 
