@@ -144,6 +144,27 @@ etg_status etg_debug_expand_replay(etg_graph *g, int alg, uint32_t source, uint3
                                    uint32_t tune, int reps, uint32_t *d_label, uint32_t *d_saved,
                                    float *ms, uint64_t *edges, uint32_t *n_active);
 
+/* ---- Step-wise driving (1-D vertex-range partitions over several GPUs, Sec.
+ * "Multi-GPU" of DESIGN.md).  A partition's handle is loaded with the
+ * rank's destination-partitioned CSR: all n source rows, only the edges whose
+ * destination lies in the rank's owned range, global vertex ids.  Labels and
+ * the active-set bitmap are full-size (n) on every rank.  Protocol:
+ *   etg_step_begin -> while (n_active) { etg_step_expand; exchange;
+ *   etg_step_scan } -> etg_step_end,
+ * where "exchange" makes every rank's bitmap (etg_bitmap_layout: nwords uint32
+ * words at offset_bytes into the workspace) the OR of all ranks' bitmaps and,
+ * for SSSP/CC/SSWP, every rank's labels the min (SSWP: max) over ranks.
+ * n_active is the number of vertices activated (bitmap bits consumed by the
+ * scan); it is identical on every rank after an exchange, so all ranks leave
+ * the loop together (a rank whose compacted set is empty expands nothing).
+ * etg_step_begin already runs the first scan (the initial active set). */
+etg_status etg_step_begin(etg_graph *g, int alg, uint32_t source, uint32_t *d_label,
+                          uint32_t *n_active);
+etg_status etg_step_expand(etg_graph *g);
+etg_status etg_step_scan(etg_graph *g, uint32_t *n_active);
+etg_status etg_step_end(etg_graph *g, etg_stats *st_or_null);
+etg_status etg_bitmap_layout(etg_graph *g, size_t *offset_bytes, uint32_t *nwords);
+
 /* Release a handle (does not free the borrowed device memory). */
 void etg_free(etg_graph *g);
 

@@ -82,6 +82,11 @@ def lib():
             "etg_status_str": (ctypes.c_char_p, [st]),
             "etg_last_error": (ctypes.c_char_p, []),
             "etg_kernel_launches": (u64, []),
+            "etg_step_begin": (st, [p, ctypes.c_int, u32, p, ctypes.POINTER(u32)]),
+            "etg_step_expand": (st, [p]),
+            "etg_step_scan": (st, [p, ctypes.POINTER(u32)]),
+            "etg_step_end": (st, [p, p]),
+            "etg_bitmap_layout": (st, [p, ctypes.POINTER(sz), ctypes.POINTER(u32)]),
             "etg_debug_expand_replay": (st, [p, ctypes.c_int, u32, u32, u32, ctypes.c_int, p, p,
                                              ctypes.POINTER(ctypes.c_float), ctypes.POINTER(u64),
                                              ctypes.POINTER(u32)]),

@@ -137,6 +137,9 @@ struct etg_graph {
     Ctl *h_ctl = nullptr;                 // pinned host mirror for readback
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     cudaEvent_t pev[3] = {nullptr, nullptr, nullptr};   // ETG_PROFILE: scan / expand brackets
+    int step_alg = -1;                    // algorithm of the step-wise (distributed) run
+    uint64_t step_launches = 0;
+    uint64_t step_acts = 0;               // activations counted so far (cumulative)
     cudaGraphExec_t exec[4] = {nullptr, nullptr, nullptr, nullptr};
     cudaGraph_t graph[4] = {nullptr, nullptr, nullptr, nullptr};
 };
@@ -368,6 +371,64 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
         st->edges_reached = 0;
         st->ms = ms;
     }
+    return ETG_OK;
+}
+
+
+// --------------------------------------------------------------------------- //
+// Step-wise driving (multi-GPU partitions, A6 exchanged between steps): the
+// caller runs begin, then { expand; exchange Q (and labels); scan } while the
+// active set is non-empty, then end.  Same kernels as the fused loop.
+// --------------------------------------------------------------------------- //
+template <class OffT>
+etg_status step_scan_impl(etg_graph *g, uint32_t *n_active);
+
+template <class OffT>
+etg_status step_begin_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, uint32_t *n_active,
+                           int skip_scan) {
+    Dev<OffT> d = make_dev<OffT>(g);
+    cudaStream_t s = g->stream;
+    ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, label, source);
+    void *iargs[] = {&d, &label, &source};
+    ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), iargs, 0, s));
+    g->step_launches = 2;
+    g->step_alg = alg;
+    g->step_acts = 0;
+    if (!skip_scan) return step_scan_impl<OffT>(g, n_active);
+    ETG_CU(cudaStreamSynchronize(s));
+    *n_active = 0;
+    return ETG_OK;
+}
+
+template <class OffT>
+etg_status step_scan_impl(etg_graph *g, uint32_t *n_active) {
+    Dev<OffT> d = make_dev<OffT>(g);
+    cudaStream_t s = g->stream;
+    cudaGraphConditionalHandle none = 0;
+    int zero = 0;
+    void *scan_args[] = {&d, &none, &zero};
+    ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, g->step_alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+    g->step_launches += 1;
+    ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    ETG_CU(cudaStreamSynchronize(s));
+    ETG_CU(cudaGetLastError());
+    // vertices activated (bits consumed) by this scan: the same on every rank
+    *n_active = (uint32_t)(g->h_ctl->activations - g->step_acts);
+    g->step_acts = g->h_ctl->activations;
+    return ETG_OK;
+}
+
+template <class OffT>
+etg_status step_expand_impl(etg_graph *g) {
+    Dev<OffT> d = make_dev<OffT>(g);
+    Launch ex;
+    etg_status rc = expand_launch<OffT>(g, g->step_alg, ex);
+    if (rc != ETG_OK) return rc;
+    uint32_t cap_e = g->p.ts * g->p.K;
+    void *exp_args[] = {&d, &cap_e};
+    if (g->p.warp) exp_args[1] = nullptr;
+    ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, g->stream));
+    g->step_launches += 1;
     return ETG_OK;
 }
 
@@ -606,6 +667,51 @@ etg_status etg_debug_expand_replay(etg_graph *g, int alg, uint32_t source, uint3
     if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "no weights");
     return g->p.u64 ? replay_impl<uint64_t>(g, alg, source, depth, tune, reps, d_label, d_saved, ms, edges, n_active)
                     : replay_impl<uint32_t>(g, alg, source, depth, tune, reps, d_label, d_saved, ms, edges, n_active);
+}
+
+etg_status etg_step_begin(etg_graph *g, int alg, uint32_t source, uint32_t *d_label, uint32_t *n_active) {
+    if (!g || !d_label || !n_active) return fail(ETG_EINVAL, "NULL argument");
+    if (alg < 0 || alg > 3) return fail(ETG_EINVAL, "alg must be 0..3");
+    if (alg != ALG_CC && source >= g->n) return fail(ETG_EINVAL, "source >= n");
+    if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "graph loaded without weights");
+    if (alg == ALG_CC && !(g->flags & ETG_SYMMETRIC)) return fail(ETG_ENOTSYM, "etg_cc needs ETG_SYMMETRIC");
+    if (g->n == 0) { *n_active = 0; return ETG_OK; }
+    return g->p.u64 ? step_begin_impl<uint64_t>(g, alg, source, d_label, n_active, 0)
+                    : step_begin_impl<uint32_t>(g, alg, source, d_label, n_active, 0);
+}
+
+etg_status etg_step_expand(etg_graph *g) {
+    if (!g || g->step_alg < 0) return fail(ETG_EINVAL, "no step-wise run in progress");
+    return g->p.u64 ? step_expand_impl<uint64_t>(g) : step_expand_impl<uint32_t>(g);
+}
+
+etg_status etg_step_scan(etg_graph *g, uint32_t *n_active) {
+    if (!g || !n_active || g->step_alg < 0) return fail(ETG_EINVAL, "no step-wise run in progress");
+    return g->p.u64 ? step_scan_impl<uint64_t>(g, n_active) : step_scan_impl<uint32_t>(g, n_active);
+}
+
+etg_status etg_step_end(etg_graph *g, etg_stats *st) {
+    if (!g || g->step_alg < 0) return fail(ETG_EINVAL, "no step-wise run in progress");
+    ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g->stream));
+    ETG_CU(cudaStreamSynchronize(g->stream));
+    g_launches += g->step_launches;
+    g->step_alg = -1;
+    if (st) {
+        memset(st, 0, sizeof(*st));
+        st->iterations = g->h_ctl->iterations;
+        st->activations = g->h_ctl->activations;
+        st->frontier_total = g->h_ctl->frontier;
+        st->shadows = g->h_ctl->shadows;
+        st->edges_processed = g->h_ctl->edges;
+    }
+    return ETG_OK;
+}
+
+etg_status etg_bitmap_layout(etg_graph *g, size_t *offset_bytes, uint32_t *nwords) {
+    if (!g || !offset_bytes || !nwords) return fail(ETG_EINVAL, "NULL argument");
+    *offset_bytes = g->L.Q;
+    *nwords = g->L.nwords;
+    return ETG_OK;
 }
 
 void etg_free(etg_graph *g) {

@@ -1,0 +1,192 @@
+"""Multi-GPU traversal: 1-D destination-range partition + per-iteration exchange.
+
+Design:
+
+* vertex range R_g = [lo_g, hi_g) per rank, boundaries multiples of 32 (one
+  bitmap word has one owner), chosen so every rank owns about the same number
+  of IN-edges (the work of a push relaxation lands on the destination);
+* rank g holds E_g = {(u, v) in E : v in R_g} as a CSR over all n sources
+  (global ids) -- relaxations on rank g only ever touch owned vertices;
+* every rank expands the same, replicated, compacted active set (UDC over its
+  own sub-rows, so a hub's edges are split ~deg/P per rank), marks improved
+  owned vertices in its bitmap, then the exchange makes the bitmaps the union
+  (ranges are word-disjoint, so an integer all-reduce SUM is the OR) and, for
+  SSSP/CC/SSWP, the labels the element-wise best (MIN; MAX for SSWP): a
+  non-owner's copy is the owner's value from an earlier exchange, never better
+  than the owner's current one.  BFS exchanges the bitmap only -- each rank's
+  scan writes the depth of every vertex of the new active set.
+* termination: the compacted active-set size after the exchange is identical
+  on every rank (same bitmap), so all ranks leave the loop together.
+
+Only argument marshalling and the collective calls are in Python; every step of
+the traversal runs in libetg.so (etg_step_begin / etg_step_expand /
+etg_step_scan / etg_step_end).  The collective is torch.distributed (NCCL over
+NVLink on the GPU box); ``LoopbackGroup`` runs P partitions on one GPU for
+tests.
+"""
+from __future__ import annotations
+
+import ctypes
+from typing import Callable, List, Optional, Sequence
+
+import torch
+
+from . import (BFS, CC, SSSP, SSWP, EtgError, Graph, Stats, _check, _ptr, lib)
+
+SIGN = -(1 << 31)   # xor with this maps uint32 order onto int32 order
+
+
+# --------------------------------------------------------------------------- #
+# partitioning (host logic; torch ops on whatever device the CSR lives on)
+# --------------------------------------------------------------------------- #
+def partition_ranges(off: torch.Tensor, col: torch.Tensor, n: int, P: int, align: int = 32) -> List[int]:
+    """Boundaries lo_0 = 0 < ... < lo_P = n, multiples of `align` (except n),
+    balancing in-edge counts.  Returns the P + 1 boundaries."""
+    if P < 1:
+        raise ValueError("P >= 1")
+    indeg = torch.bincount(col.to(torch.int64), minlength=n)
+    cum = torch.cumsum(indeg, 0)
+    m = int(cum[-1]) if n else 0
+    bounds = [0]
+    for g in range(1, P):
+        target = (m * g) // P
+        v = int(torch.searchsorted(cum, torch.tensor(target, device=cum.device)))
+        v = (v + align // 2) // align * align
+        v = min(max(v, bounds[-1]), n)
+        bounds.append(v)
+    bounds.append(n)
+    return bounds
+
+
+def partition_csr(off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor], n: int,
+                  lo: int, hi: int):
+    """The rank's destination-partitioned CSR: rows = all n sources, edges with
+    destination in [lo, hi), CSR order kept, global ids."""
+    off = off.to(torch.int64)
+    col = col.to(torch.int64)
+    keep = (col >= lo) & (col < hi)
+    src = torch.repeat_interleave(torch.arange(n, device=off.device), off[1:] - off[:-1])
+    src = src[keep]
+    cnt = torch.bincount(src, minlength=n)
+    loff = torch.zeros(n + 1, dtype=torch.int64, device=off.device)
+    loff[1:] = torch.cumsum(cnt, 0)
+    return loff, col[keep], (None if w is None else w.to(torch.int64)[keep])
+
+
+# --------------------------------------------------------------------------- #
+# collectives
+# --------------------------------------------------------------------------- #
+class TorchDistGroup:
+    """all_reduce over a torch.distributed process group (NCCL on GPUs, gloo on CPUs)."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        self.dist = dist
+        self.group = group
+
+    def allreduce(self, tensors: Sequence[torch.Tensor], op: str) -> None:
+        ops = {"sum": self.dist.ReduceOp.SUM, "min": self.dist.ReduceOp.MIN,
+               "max": self.dist.ReduceOp.MAX}
+        assert len(tensors) == 1
+        self.dist.all_reduce(tensors[0], op=ops[op], group=self.group)
+
+
+class LoopbackGroup:
+    """P 'ranks' in one process (one GPU): all_reduce over a list of tensors."""
+
+    def allreduce(self, tensors: Sequence[torch.Tensor], op: str) -> None:
+        acc = tensors[0].clone()
+        for t in tensors[1:]:
+            if op == "sum":
+                acc += t
+            elif op == "min":
+                acc = torch.minimum(acc, t)
+            else:
+                acc = torch.maximum(acc, t)
+        for t in tensors:
+            t.copy_(acc)
+
+
+# --------------------------------------------------------------------------- #
+# engines: the CUDA handle (product) behind a small step interface
+# --------------------------------------------------------------------------- #
+class CudaEngine:
+    """One partition on one GPU, driven step-wise through the C ABI."""
+
+    def __init__(self, graph: Graph):
+        self.g = graph
+        off = ctypes.c_size_t()
+        nw = ctypes.c_uint32()
+        _check(lib().etg_bitmap_layout(graph._h, ctypes.byref(off), ctypes.byref(nw)), "etg_bitmap_layout")
+        self.q = graph.workspace[off.value: off.value + 4 * nw.value].view(torch.int32)
+        self.labels = torch.empty(graph.n, dtype=torch.int32, device=graph.device)
+
+    def begin(self, alg: int, source: int) -> int:
+        na = ctypes.c_uint32()
+        _check(lib().etg_step_begin(self.g._h, alg, source, _ptr(self.labels), ctypes.byref(na)),
+               "etg_step_begin")
+        return int(na.value)
+
+    def expand(self) -> None:
+        _check(lib().etg_step_expand(self.g._h), "etg_step_expand")
+
+    def scan(self) -> int:
+        na = ctypes.c_uint32()
+        _check(lib().etg_step_scan(self.g._h, ctypes.byref(na)), "etg_step_scan")
+        return int(na.value)
+
+    def end(self) -> Stats:
+        st = Stats()
+        _check(lib().etg_step_end(self.g._h, ctypes.byref(st)), "etg_step_end")
+        return st
+
+
+def _exchange(engines, group, alg: int) -> None:
+    """Union of the bitmaps; best labels (SSSP/CC: min, SSWP: max) -- see module doc."""
+    group.allreduce([e.q for e in engines], "sum")
+    if alg != BFS:
+        labs = [e.labels for e in engines]
+        for t in labs:
+            t.bitwise_xor_(SIGN)            # uint32 order -> int32 order
+        group.allreduce(labs, "max" if alg == SSWP else "min")
+        for t in labs:
+            t.bitwise_xor_(SIGN)
+
+
+def run_partitions(engines, group, alg: int, source: int = 0):
+    """Drive P engines in lockstep (all in this process: loopback), or ONE
+    engine of this rank (torch.distributed: the other ranks run the same
+    loop).  Returns (labels of engines[0], summed stats, iterations)."""
+    n_act = [e.begin(alg, source) for e in engines]
+    while n_act[0] > 0:
+        for e in engines:
+            e.expand()
+        _exchange(engines, group, alg)
+        n_act = [e.scan() for e in engines]
+        if len(set(n_act)) != 1:
+            raise EtgError(f"ranks disagree on the active-set size: {n_act}")
+    stats = [e.end() for e in engines]
+    total = Stats()
+    total.iterations = stats[0].iterations
+    for f in ("activations", "frontier_total", "shadows", "edges_processed"):
+        setattr(total, f, sum(getattr(s, f) for s in stats))
+    return engines[0].labels, total
+
+
+class DistGraph:
+    """This rank's partition of a graph, driven over a torch.distributed group."""
+
+    def __init__(self, off, col, w, n: int, rank: int, world: int, *, K: int = 32, flags: int = 0,
+                 symmetric: bool = False, device="cuda", group=None, bounds=None):
+        from . import csr_to_device
+        self.n, self.rank, self.world = n, rank, world
+        self.bounds = bounds if bounds is not None else partition_ranges(off, col, n, world)
+        lo, hi = self.bounds[rank], self.bounds[rank + 1]
+        loff, lcol, lw = partition_csr(off, col, w, n, lo, hi)
+        o, c, ww, fl = csr_to_device(loff, lcol, lw, device=device)
+        self.graph = Graph(o, c, ww, n=n, K=K, flags=flags | fl, symmetric=symmetric)
+        self.engine = CudaEngine(self.graph)
+        self.group = TorchDistGroup(group)
+
+    def run(self, alg: int, source: int = 0):
+        return run_partitions([self.engine], self.group, alg, source)

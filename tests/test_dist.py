@@ -1,0 +1,99 @@
+"""Multi-rank path: partitioning and the exchange driver, on the CPU.
+
+* partition properties (every edge in exactly one part, word-aligned ranges,
+  in-edge balance);
+* the driver with P in-process ranks (LoopbackGroup) and with world_size 2
+  over gloo (torch.distributed, 127.0.0.1), each rank a test-only numpy step
+  engine (tests/etg_mock_engine.py) -- labels must equal the oracle's.
+The CUDA engine through the same driver is covered by tests/test_gpu_dist.py.
+"""
+import os
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import graphgen as gg
+import oracle
+from etg_mock_engine import MockEngine
+from paper_conf_ipps_wangzlg19_b200 import dist as edist
+
+ALGS = {"bfs": 0, "sssp": 1, "cc": 2, "sswp": 3}
+
+
+def expected(alg, g, s):
+    off, col, w = g.numpy()
+    if alg == "bfs":
+        return oracle.bfs(off, col, s)
+    if alg == "sssp":
+        return oracle.sssp(off, col, w, s)
+    if alg == "sswp":
+        return oracle.sswp(off, col, w, s)
+    return oracle.cc(off, col)
+
+
+def make_parts(g, P):
+    bounds = edist.partition_ranges(g.off, g.col, g.n, P)
+    parts = []
+    for r in range(P):
+        loff, lcol, lw = edist.partition_csr(g.off, g.col, g.w, g.n, bounds[r], bounds[r + 1])
+        parts.append(MockEngine(loff.numpy(), lcol.numpy(), None if lw is None else lw.numpy(), g.n))
+    return bounds, parts
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 5])
+def test_partition_properties(P):
+    g = gg.make("T12")
+    bounds = edist.partition_ranges(g.off, g.col, g.n, P)
+    assert bounds[0] == 0 and bounds[-1] == g.n and len(bounds) == P + 1
+    assert all(b % 32 == 0 for b in bounds[:-1]) and all(a <= b for a, b in zip(bounds, bounds[1:]))
+    seen = 0
+    indeg = np.bincount(g.col.numpy(), minlength=g.n)
+    for r in range(P):
+        loff, lcol, lw = edist.partition_csr(g.off, g.col, g.w, g.n, bounds[r], bounds[r + 1])
+        assert loff.shape[0] == g.n + 1 and int(loff[-1]) == lcol.shape[0]
+        assert torch.all((lcol >= bounds[r]) & (lcol < bounds[r + 1]))
+        seen += lcol.shape[0]
+        share = indeg[bounds[r]:bounds[r + 1]].sum() / g.m
+        assert abs(share - 1 / P) < 0.05
+    assert seen == g.m
+
+
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "cc", "sswp"])
+@pytest.mark.parametrize("P", [2, 3])
+def test_loopback_driver_matches_oracle(alg, P):
+    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
+    s = gg.first_source(g)
+    _, parts = make_parts(g, P)
+    labels, st = edist.run_partitions(parts, edist.LoopbackGroup(), ALGS[alg], s)
+    np.testing.assert_array_equal(labels.numpy().view(np.uint32), expected(alg, g, s))
+    if alg == "bfs":
+        assert st.edges_processed == int(np.diff(g.off.numpy())[expected(alg, g, s) != oracle.INF].sum())
+
+
+def _gloo_worker(rank, world, port, alg, out):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
+    s = gg.first_source(g)
+    bounds = edist.partition_ranges(g.off, g.col, g.n, world)
+    loff, lcol, lw = edist.partition_csr(g.off, g.col, g.w, g.n, bounds[rank], bounds[rank + 1])
+    eng = MockEngine(loff.numpy(), lcol.numpy(), None if lw is None else lw.numpy(), g.n)
+    labels, st = edist.run_partitions([eng], edist.TorchDistGroup(), ALGS[alg], s)
+    torch.save(labels, out + f".{rank}")
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "cc"])
+def test_gloo_world2_matches_oracle(alg, tmp_path):
+    port = 29500 + (os.getpid() % 1000) + ALGS[alg]
+    out = str(tmp_path / "labels")
+    mp.spawn(_gloo_worker, args=(2, port, alg, out), nprocs=2, join=True)
+    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
+    exp = expected(alg, g, gg.first_source(g))
+    for r in range(2):
+        got = torch.load(out + f".{r}").numpy().view(np.uint32)
+        np.testing.assert_array_equal(got, exp)

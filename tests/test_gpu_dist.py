@@ -1,0 +1,60 @@
+"""The partitioned (multi-GPU) path with the CUDA engine, P partitions on one
+GPU driven in lockstep by the same driver the NCCL ranks use (LoopbackGroup):
+the assembled labels must equal the oracle's bit for bit."""
+import numpy as np
+import pytest
+import torch
+
+import graphgen as gg
+import oracle
+
+pytestmark = pytest.mark.gpu
+etg = pytest.importorskip("paper_conf_ipps_wangzlg19_b200")
+from paper_conf_ipps_wangzlg19_b200 import dist as edist  # noqa: E402
+
+ALG = {"bfs": etg.BFS, "sssp": etg.SSSP, "cc": etg.CC, "sswp": etg.SSWP}
+
+
+def engines(g, P, K=32, flags=0):
+    bounds = edist.partition_ranges(g.off, g.col, g.n, P)
+    out = []
+    for r in range(P):
+        loff, lcol, lw = edist.partition_csr(g.off, g.col, g.w, g.n, bounds[r], bounds[r + 1])
+        o, c, w, fl = etg.csr_to_device(loff, lcol, lw, device="cuda")
+        G = etg.Graph(o, c, w, n=g.n, K=K, flags=flags | fl, symmetric=g.symmetric)
+        out.append(edist.CudaEngine(G))
+    return out
+
+
+def expected(alg, g, s):
+    off, col, w = g.numpy()
+    return {"bfs": lambda: oracle.bfs(off, col, s), "sssp": lambda: oracle.sssp(off, col, w, s),
+            "sswp": lambda: oracle.sswp(off, col, w, s), "cc": lambda: oracle.cc(off, col)}[alg]()
+
+
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "cc", "sswp"])
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_partitioned_c1(alg, P):
+    g = gg.make("C1", symmetric=(alg == "cc"), weights=(alg != "cc"))
+    s = gg.sample_sources(g, 1, P)[0]
+    labels, st = edist.run_partitions(engines(g, P), edist.LoopbackGroup(), ALG[alg], s)
+    np.testing.assert_array_equal(etg.to_u32_numpy(labels), expected(alg, g, s))
+
+
+def test_partitioned_bfs_work_is_split():
+    """Every edge of the activatable subgraph is relaxed on exactly one rank."""
+    g = gg.make("T14", weights=False)
+    s = gg.first_source(g)
+    labels, st = edist.run_partitions(engines(g, 4), edist.LoopbackGroup(), etg.BFS, s)
+    exp = expected("bfs", g, s)
+    deg = np.diff(g.off.numpy())
+    assert st.edges_processed == int(deg[exp != etg.INF].sum())
+    np.testing.assert_array_equal(etg.to_u32_numpy(labels), exp)
+
+
+def test_partitioned_k_and_flags():
+    g = gg.make("LJ-small")
+    s = gg.sample_sources(g, 1, 9)[0]
+    for K, flags in ((8, 0), (1024, 0), (32, etg.NO_UDC)):
+        labels, _ = edist.run_partitions(engines(g, 3, K, flags), edist.LoopbackGroup(), etg.SSSP, s)
+        np.testing.assert_array_equal(etg.to_u32_numpy(labels), expected("sssp", g, s))
