@@ -314,7 +314,7 @@ CONFIGS = {
     "C2": dict(kind="rmat", scale=22, edge_factor=16, seed=22),
     # C3: LiveJournal-shaped Chung-Lu (4.8M vertices, ~69M edges)
     "C3": dict(kind="chunglu", n=4_800_000, m_target=69_000_000, alpha_out=1.9,
-               dmax_out=20_000, alpha_in=2.0, dmax_in=14_000, oversample=1.06, seed=3),
+               dmax_out=20_000, alpha_in=2.0, dmax_in=14_000, oversample=1.03, seed=3),
     # C4: Twitter-shaped Chung-Lu (41.6M vertices, ~1.47B edges)
     "C4": dict(kind="chunglu", n=41_600_000, m_target=1_470_000_000, alpha_out=1.7,
                dmax_out=3_000_000, alpha_in=2.1, dmax_in=300_000, oversample=1.16, seed=41),

@@ -1,0 +1,47 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py
+times (CUDA-graph loop, K = 32, default flags): C2 (the bench workload) and
+C3 (LiveJournal-shaped, UDC on and off).  The single-threaded oracle finishes
+these in seconds, so the comparison is complete (all n labels), not sampled."""
+import numpy as np
+import pytest
+import torch
+
+import graphgen as gg
+import oracle
+from etg_testutil import to_etg
+
+pytestmark = pytest.mark.gpu
+etg = pytest.importorskip("paper_conf_ipps_wangzlg19_b200")
+U32 = etg.to_u32_numpy
+
+
+@pytest.fixture(scope="module")
+def c2():
+    return gg.make("C2", device="cuda")
+
+
+def test_c2_bfs_sssp_sswp(c2):
+    off, col, w = c2.to("cpu").numpy()
+    G = to_etg(c2)
+    for s in gg.sample_sources(c2, 2, 4242):
+        np.testing.assert_array_equal(U32(G.bfs(s)[0]), oracle.bfs(off, col, s))
+        np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
+    s = gg.first_source(c2)
+    np.testing.assert_array_equal(U32(G.sswp(s)[0]), oracle.sswp(off, col, w, s))
+
+
+def test_c2_cc():
+    gs = gg.make("C2", device="cuda", symmetric=True, weights=False)
+    soff, scol, _ = gs.to("cpu").numpy()
+    G = to_etg(gs, symmetric=True)
+    np.testing.assert_array_equal(U32(G.cc()[0]), oracle.cc(soff, scol))
+
+
+@pytest.mark.parametrize("flags", [0, 2])
+def test_c3_lj_shaped(flags):
+    g = gg.make("C3", device="cuda")
+    off, col, w = g.to("cpu").numpy()
+    G = to_etg(g, flags=flags)
+    s = gg.first_source(g)
+    np.testing.assert_array_equal(U32(G.bfs(s)[0]), oracle.bfs(off, col, s))
+    np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
