@@ -85,7 +85,7 @@ Params derive(const etg_options *opt, uint32_t tune) {
 }
 
 struct Layout {
-    size_t Q, F, B, D, S, tile_first, st_flag, st_agg, st_inc, ctl, total;
+    size_t Q, snap, F, B, D, S, tile_first, st_flag, st_agg, st_inc, ctl, total;
     uint32_t nwords;
 };
 
@@ -104,6 +104,7 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
     const uint64_t tile_words = kScanV / 32;
     L.nwords = (uint32_t)((words + tile_words - 1) / tile_words * tile_words);
     L.Q = take(4ull * L.nwords);
+    L.snap = take(4 * (n + 1));
     L.F = take(4 * (n + 1));
     L.B = take((p.u64 ? 8 : 4) * (n + 1));
     L.D = take(4 * (n + 1));
@@ -154,6 +155,7 @@ Dev<OffT> make_dev(const etg_graph *g) {
     d.w = g->w;
     d.Q = reinterpret_cast<uint32_t *>(g->ws + g->L.Q);
     d.nwords = g->L.nwords;
+    d.snap = reinterpret_cast<uint32_t *>(g->ws + g->L.snap);
     d.F = reinterpret_cast<uint32_t *>(g->ws + g->L.F);
     d.B = reinterpret_cast<OffT *>(g->ws + g->L.B);
     d.D = reinterpret_cast<uint32_t *>(g->ws + g->L.D);
@@ -528,6 +530,8 @@ etg_status replay_impl(etg_graph *g, int alg, uint32_t source, uint32_t depth, u
     float total = 0.f;
     for (int r = 0; r < reps; ++r) {
         ETG_CU(cudaMemcpyAsync(label, saved, 4ull * g->n, cudaMemcpyDeviceToDevice, s));
+        if (alg != ALG_BFS)   // the pre-filter snapshot equals the labels at an iteration start
+            ETG_CU(cudaMemcpyAsync(d.snap, saved, 4ull * g->n, cudaMemcpyDeviceToDevice, s));
         ETG_CU(cudaMemsetAsync(d.Q, 0, 4ull * g->L.nwords, s));
         *g->h_ctl = snap;
         ETG_CU(cudaMemcpyAsync(g->ctl, g->h_ctl, sizeof(Ctl), cudaMemcpyHostToDevice, s));

@@ -80,6 +80,7 @@ struct Dev {
     const uint32_t *col;
     const uint32_t *w;
     uint32_t *Q;                // next-active-set bitmap (nwords words, zero between uses)
+    uint32_t *snap;             // labels at the start of the iteration (SSSP/CC/SSWP pre-filter)
     uint32_t *F;                // compacted active set (vertex ids, ascending)
     OffT *B;                    // off[F[k]]
     uint32_t *D;                // out-degree of F[k] (> 0)
@@ -102,10 +103,11 @@ constexpr uint32_t kTuneFilterL1 = 1u;    // pre-filter label loads cached in L1
 constexpr uint32_t kTuneNoGather = 16u;   // skip the label gather and the commit
 constexpr uint32_t kTuneNoCommit = 32u;   // gather labels but never commit (counts passes)
 constexpr uint32_t kTuneBitOnly = 64u;    // commit = red.or of the bitmap only
-constexpr uint32_t kTuneHashU = 128u;     // targets from a hash of x (no column loads)
-constexpr uint32_t kTuneNoOwner = 256u;   // column index = tile base + x (no owner logic)
 constexpr uint32_t kTuneNoPrefetch = 512u; // no L2 prefetch of the next tile's segments
 constexpr uint32_t kTuneStatic = 1024u;    // static round-robin tile schedule
+constexpr uint32_t kTuneRedMinOnly = 2048u; // commit: label reduction only (no bitmap mark)
+constexpr uint32_t kTuneRedOrOnly = 4096u;  // commit: bitmap mark only (no label reduction)
+constexpr uint32_t kTuneNoHint = 8192u;     // commit reductions without the L2 policy
 
 // ------------------------------------------------------------------------- //
 // small device helpers
@@ -267,6 +269,7 @@ __global__ __launch_bounds__(kBlock) void init_kernel(Dev<OffT> d, uint32_t *lab
         else if (ALG == ALG_SSWP) lab = (v == source) ? kInf : 0u;
         else lab = (v == source) ? 0u : kInf;
         label[v] = lab;
+        if (ALG != ALG_BFS) d.snap[v] = lab;
     }
     if (ALG == ALG_CC) {
         for (uint32_t k = blockIdx.x * kBlock + threadIdx.x; k < d.nwords; k += stride) {
@@ -406,6 +409,7 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
                 if (bits & (1u << k)) {
                     const uint32_t v = v0 + k;
                     if (BFSLAB) label[v] = new_depth;      // BFS: depth written once, on compaction
+                    else if (label) d.snap[v] = __ldcg(&label[v]);   // refresh the pre-filter snapshot
                     const uint32_t dg = (uint32_t)(o[k + 1] - o[k]);
                     const uint32_t c = udc_count<UDC>(dg, d.K);
                     if (c) {
@@ -788,54 +792,41 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
         const uint32_t E = __shfl_sync(kFull, incl, 31);
         my_edges += E;
         uint32_t owner = 0xFFFFFFFFu;                         // owner of the element before x0
-        // Software pipeline over batches of kR chunks (32 elements each): the
-        // column loads of batch b+1 are issued before the label gathers of
-        // batch b, so a warp always has gathers or column loads in flight.
-        uint32_t un[kR], cn[kR];
-        bool an[kR];
-        auto fetch = [&](uint32_t x0) {
+        // Batches of kR chunks of 32 elements.  The owner of element x is the
+        // number of slice starts <= x, minus one: the batch's kR words of the
+        // start mask come from kR independent OR-reductions, then a popcount
+        // prefix -- no serial dependency between the chunks of a batch.
+        for (uint32_t x0 = 0; x0 < E; x0 += 32u * kR) {
+            uint32_t u[kR], c[kR], cur[kR], wv[kR];
+            bool act[kR];
+            const uint32_t pos = o - x0;                      // this lane's slice start in the batch
+            const bool in_win = sh.len && pos < 32u * kR;
+            uint32_t wm[kR];
+#pragma unroll
+            for (int r = 0; r < kR; ++r)
+                wm[r] = __reduce_or_sync(kFull, (in_win && (pos >> 5) == (uint32_t)r) ? (1u << (pos & 31)) : 0u);
 #pragma unroll
             for (int r = 0; r < kR; ++r) {
-                const uint32_t cx = x0 + 32u * r;            // chunk start
-                const uint32_t pos = o - cx;                  // this lane's slice start in the chunk
-                uint32_t sm = 0;
-                if (!(d.tune & kTuneNoOwner))
-                    sm = __reduce_or_sync(kFull, (sh.len && pos < 32u) ? (1u << pos) : 0u);
-                const uint32_t own = owner + __popc(sm & lt_eq);
-                owner += __popc(sm);
+                const uint32_t own = owner + __popc(wm[r] & lt_eq);
+                owner += __popc(wm[r]);
                 const uint32_t src = own & 31u;
-                const OffT dl = (d.tune & kTuneNoOwner) ? __shfl_sync(kFull, delta, 0) : __shfl_sync(kFull, delta, src);
+                const OffT dl = __shfl_sync(kFull, delta, src);
                 const uint32_t ll = (ALG == ALG_BFS) ? level : __shfl_sync(kFull, lab, src);
-                const uint32_t x = cx + lane;
-                an[r] = x < E;
-                un[r] = 0;
-                cn[r] = ll;
-                if (an[r]) {
+                const uint32_t x = x0 + 32u * r + lane;
+                act[r] = x < E;
+                u[r] = 0;
+                c[r] = ll;
+                wv[r] = 0;
+                if (act[r]) {
                     const OffT e = dl + (OffT)x;
-                    if (d.tune & kTuneHashU) {
-                        uint32_t h = (uint32_t)e * 0x9E3779B1u;
-                        h ^= h >> 15;
-                        h *= 0x85EBCA77u;
-                        h ^= h >> 13;
-                        un[r] = h % d.n;
-                    } else {
-                        un[r] = ld_stream(&d.col[e], stream);
-                    }
-                    if (kW) cn[r] = candidate<ALG>(ll, ld_stream(&d.w[e], stream));
+                    u[r] = ld_stream(&d.col[e], stream);
+                    if (kW) wv[r] = ld_stream(&d.w[e], stream);
                 }
             }
-        };
-        fetch(0);
-        for (uint32_t x0 = 0; x0 < E; x0 += 32u * kR) {
-            uint32_t u[kR], c[kR], cur[kR];
-            bool act[kR];
+            if (kW) {
 #pragma unroll
-            for (int r = 0; r < kR; ++r) {
-                u[r] = un[r];
-                c[r] = cn[r];
-                act[r] = an[r];
+                for (int r = 0; r < kR; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
             }
-            if (x0 + 32u * kR < E) fetch(x0 + 32u * kR);      // next batch's column loads
             if (d.tune & kTuneNoGather) {                     // replay experiment
                 uint32_t x = 0;
 #pragma unroll
@@ -843,9 +834,13 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
                 if (x == 0x9E3779B9u) Q[0] = x;
                 continue;
             }
+            // pre-filter: BFS reads the labels (written only by the scan); the
+            // others read the iteration-start snapshot, so the gathers and the
+            // red.min/max commits never touch the same lines (R-4, R-6)
+            const uint32_t *filt = (ALG == ALG_BFS) ? label : d.snap;
 #pragma unroll
             for (int r = 0; r < kR; ++r)
-                cur[r] = act[r] ? (l1 ? ld_ca(&label[u[r]]) : ld_label(&label[u[r]], keep)) : 0u;
+                cur[r] = act[r] ? (l1 ? ld_ca(&filt[u[r]]) : ld_label(&filt[u[r]], keep)) : 0u;
             if (d.tune & kTuneNoCommit) {                     // replay experiment: count passes
                 uint32_t x = 0;
 #pragma unroll
@@ -857,6 +852,21 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
 #pragma unroll
                 for (int r = 0; r < kR; ++r)
                     if (act[r] && improves<ALG>(c[r], cur[r])) red_or(&Q[u[r] >> 5], 1u << (u[r] & 31), keep);
+                continue;
+            }
+            if (d.tune & (kTuneRedMinOnly | kTuneRedOrOnly | kTuneNoHint)) {   // replay experiments
+#pragma unroll
+                for (int r = 0; r < kR; ++r) {
+                    if (!(act[r] && improves<ALG>(c[r], cur[r]))) continue;
+                    if (d.tune & kTuneNoHint) {
+                        atomicMin(&label[u[r]], c[r]);
+                        atomicOr(&Q[u[r] >> 5], 1u << (u[r] & 31));
+                    } else if (d.tune & kTuneRedMinOnly) {
+                        red_min(&label[u[r]], c[r], keep);
+                    } else {
+                        red_or(&Q[u[r] >> 5], 1u << (u[r] & 31), keep);
+                    }
+                }
                 continue;
             }
 #pragma unroll

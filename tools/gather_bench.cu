@@ -20,7 +20,8 @@ __global__ void gather(const uint32_t *__restrict__ idx, uint32_t *lab, uint64_t
             if (MODE == 0) v[r] = __ldcg(&lab[u[r]]);
             else if (MODE == 1) asm volatile("ld.global.ca.u32 %0, [%1];" : "=r"(v[r]) : "l"(&lab[u[r]]));
             else if (MODE == 2) v[r] = __ldg(&lab[u[r]]);
-            else v[r] = atomicMin(&lab[u[r]], 7u);
+            else if (MODE == 3) v[r] = atomicMin(&lab[u[r]], 7u);
+            else { asm volatile("red.relaxed.gpu.global.min.u32 [%0], %1;" :: "l"(&lab[u[r]]), "r"(u[r] & 1023u) : "memory"); v[r] = 0; }
         }
 #pragma unroll
         for (int r = 0; r < R; ++r) acc += v[r];
@@ -82,6 +83,7 @@ int main(int argc, char **argv) {
         run<8, 1>("ld.ca", idx, lab, n_idx, out, sms, bps, 256);
         run<8, 2>("ld.nc", idx, lab, n_idx, out, sms, bps, 256);
         run<8, 3>("atomMin", idx, lab, n_idx, out, sms, bps, 256);
+        run<8, 4>("redMin", idx, lab, n_idx, out, sms, bps, 256);
     }
     printf("err: %s\n", cudaGetErrorString(cudaGetLastError()));
     return 0;
