@@ -60,13 +60,17 @@ typedef enum {
 enum {
     ETG_SYMMETRIC = 1u << 0,   /* caller asserts the CSR is symmetric (required by etg_cc) */
     ETG_NO_UDC = 1u << 1,      /* ablation: one work item per active vertex (K = infinity) */
-    ETG_NO_SMP = 1u << 2,      /* ablation: no shared-memory staging of neighbour segments */
+    ETG_NO_SMP = 1u << 2,      /* ablation ("w/o SMP", Sec. VI-C): no look-ahead fetch of the
+                                  next tile's neighbour segments (default: TMA bulk prefetch
+                                  into L2) */
     ETG_OFFSETS_U64 = 1u << 3, /* d_row_offsets holds uint64 (needed when m >= 2^32) */
     ETG_VALIDATE = 1u << 4,    /* etg_load_csr runs an O(n+m) device check of the CSR */
     ETG_HOST_LOOP = 1u << 5,   /* drive iterations from the host (count read back each
                                   iteration) instead of a CUDA-graph conditional while node */
-    ETG_PROFILE = 1u << 6      /* implies ETG_HOST_LOOP; CUDA events around every scan and
+    ETG_PROFILE = 1u << 6,     /* implies ETG_HOST_LOOP; CUDA events around every scan and
                                   expand launch on the handle's stream fill scan_ms/expand_ms */
+    ETG_SMP_SHARED = 1u << 7   /* SMP as literally described (L199): TMA bulk copies of the next
+                                  tile's segments into per-warp shared-memory stages (K <= 32) */
 };
 
 typedef struct {

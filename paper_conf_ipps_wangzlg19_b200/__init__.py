@@ -23,11 +23,11 @@ import torch
 __all__ = [
     "EtgError", "Stats", "Graph", "load_csr", "csr_to_device", "to_u32_numpy",
     "run_host", "host_scratch_bytes", "kernel_launches", "lib",
-    "SYMMETRIC", "NO_UDC", "NO_SMP", "OFFSETS_U64", "VALIDATE", "HOST_LOOP", "PROFILE",
+    "SYMMETRIC", "NO_UDC", "NO_SMP", "OFFSETS_U64", "VALIDATE", "HOST_LOOP", "PROFILE", "SMP_SHARED",
     "INF", "CAP", "BFS", "SSSP", "CC", "SSWP",
 ]
 
-SYMMETRIC, NO_UDC, NO_SMP, OFFSETS_U64, VALIDATE, HOST_LOOP, PROFILE = 1, 2, 4, 8, 16, 32, 64
+SYMMETRIC, NO_UDC, NO_SMP, OFFSETS_U64, VALIDATE, HOST_LOOP, PROFILE, SMP_SHARED = 1, 2, 4, 8, 16, 32, 64, 128
 INF, CAP = 0xFFFFFFFF, 0xFFFFFFFE
 BFS, SSSP, CC, SSWP = 0, 1, 2, 3
 

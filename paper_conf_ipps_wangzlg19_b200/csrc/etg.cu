@@ -55,6 +55,7 @@ struct Params {
     bool warp;  // warp-centric expand (ts = 32, registers only); else the CTA-tile kernel
     bool idx;   // per-element owner index in shared memory (needs ts*K <= kCapE)
     bool smp;
+    bool prefetch;  // warp kernel: L2 bulk prefetch of the next tile's segments
     bool u64;
 };
 
@@ -75,9 +76,14 @@ Params derive(const etg_options *opt, uint32_t tune) {
     }
     p.idx = p.udc && (uint64_t)p.ts * p.K <= kCapE;
     p.smp = p.idx && !(flags & ETG_NO_SMP);
+    p.prefetch = false;
     if (p.warp) {
+        // warp kernel: tiles of 32 shadows; SMP = per-warp TMA stages of
+        // 32 * (K + 6) words, affordable in shared memory for K <= 32
         p.ts = 32;
-        p.idx = p.smp = false;
+        p.idx = false;
+        p.smp = p.udc && (flags & ETG_SMP_SHARED) && !(flags & ETG_NO_SMP) && p.K <= 32;
+        p.prefetch = p.udc && !(flags & ETG_NO_SMP) && !p.smp;
     }
     p.ts_log2 = 0;
     while ((1u << p.ts_log2) < p.ts) ++p.ts_log2;
@@ -166,6 +172,8 @@ Dev<OffT> make_dev(const etg_graph *g) {
     d.st_inc = reinterpret_cast<unsigned long long *>(g->ws + g->L.st_inc);
     d.ctl = g->ctl;
     d.n = (uint32_t)g->n;
+    d.m = g->m;
+    d.prefetch = g->p.prefetch ? 1u : 0u;
     d.K = g->p.K;
     d.ts = g->p.ts;
     d.ts_log2 = g->p.ts_log2;
@@ -183,18 +191,20 @@ const void *expand_fn(bool udc, bool idx, bool smp) {
 }
 
 template <class OffT, int ALG>
-const void *expand_warp_fn(bool udc) {
-    return udc ? (const void *)expand_warp_kernel<OffT, ALG, true> : (const void *)expand_warp_kernel<OffT, ALG, false>;
+const void *expand_warp_fn(bool udc, bool smp) {
+    if (!udc) return (const void *)expand_warp_kernel<OffT, ALG, false, false>;
+    return smp ? (const void *)expand_warp_kernel<OffT, ALG, true, true>
+               : (const void *)expand_warp_kernel<OffT, ALG, true, false>;
 }
 
 template <class OffT>
 const void *expand_fn_alg(int alg, bool udc, bool idx, bool smp, bool warp) {
     if (warp) {
         switch (alg) {
-            case ALG_BFS: return expand_warp_fn<OffT, ALG_BFS>(udc);
-            case ALG_SSSP: return expand_warp_fn<OffT, ALG_SSSP>(udc);
-            case ALG_CC: return expand_warp_fn<OffT, ALG_CC>(udc);
-            default: return expand_warp_fn<OffT, ALG_SSWP>(udc);
+            case ALG_BFS: return expand_warp_fn<OffT, ALG_BFS>(udc, smp);
+            case ALG_SSSP: return expand_warp_fn<OffT, ALG_SSSP>(udc, smp);
+            case ALG_CC: return expand_warp_fn<OffT, ALG_CC>(udc, smp);
+            default: return expand_warp_fn<OffT, ALG_SSWP>(udc, smp);
         }
     }
     switch (alg) {
@@ -222,10 +232,15 @@ const void *scan_fn(bool udc, int alg) {
     return udc ? (const void *)udc_scan_kernel<OffT, true, false> : (const void *)udc_scan_kernel<OffT, false, false>;
 }
 
+// second argument of the expand kernels: CTA kernel -> staging capacity in
+// edges; warp kernel -> words per SMP stage array
+uint32_t expand_arg(const Params &p) { return p.warp ? 32u * (p.K + 6u) : p.ts * p.K; }
+
 size_t expand_smem(const Params &p, int alg) {
+    const bool kw = (alg == ALG_SSSP || alg == ALG_SSWP);
+    if (p.warp) return p.smp ? (size_t)kWarps * 2 * (kw ? 2 : 1) * expand_arg(p) * 4 + kWarps * 16 : 0;
     if (!p.idx) return 0;
     const size_t cap = (size_t)p.ts * p.K;
-    const bool kw = (alg == ALG_SSSP || alg == ALG_SSWP);
     return (p.smp ? cap * 4 * (kw ? 2 : 1) : 0) + cap;
 }
 
@@ -238,7 +253,7 @@ struct Launch {
 template <class OffT>
 etg_status expand_launch(etg_graph *g, int alg, Launch &out) {
     out.fn = expand_fn_alg<OffT>(alg, g->p.udc, g->p.idx, g->p.smp, g->p.warp);
-    out.smem = g->p.warp ? 0 : expand_smem(g->p, alg);
+    out.smem = expand_smem(g->p, alg);
     ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)out.smem));
     ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
     int nb = 0;
@@ -256,7 +271,7 @@ etg_status build_graph(etg_graph *g, int alg) {
     Launch ex;
     etg_status s = expand_launch<OffT>(g, alg, ex);
     if (s != ETG_OK) return s;
-    uint32_t cap_e = g->p.ts * g->p.K;
+    uint32_t cap_e = expand_arg(g->p);
     cudaGraph_t graph;
     ETG_CU(cudaGraphCreate(&graph, 0));
     cudaGraphConditionalHandle cond;
@@ -274,7 +289,6 @@ etg_status build_graph(etg_graph *g, int alg) {
     cudaGraphNode_t n_scan, n_exp;
     void *exp_args[] = {&d, &cap_e};
     memset(&kp, 0, sizeof(kp));
-    if (g->p.warp) exp_args[1] = nullptr;
     kp.func = const_cast<void *>(ex.fn);
     kp.gridDim = ex.grid;
     kp.blockDim = dim3(kBlock);
@@ -324,10 +338,9 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
         Launch ex;
         etg_status rc = expand_launch<OffT>(g, alg, ex);
         if (rc != ETG_OK) return rc;
-        uint32_t cap_e = g->p.ts * g->p.K;
+        uint32_t cap_e = expand_arg(g->p);
         void *exp_args[] = {&d, &cap_e};
-        if (g->p.warp) exp_args[1] = nullptr;
-        for (;;) {
+            for (;;) {
             // "while actSet.isNotEmpty()" (L207): read the compacted size back
             ETG_CU(cudaMemcpyAsync(&g->h_ctl->nF, &g->ctl->nF, 4, cudaMemcpyDeviceToHost, s));
             ETG_CU(cudaStreamSynchronize(s));
@@ -426,9 +439,8 @@ etg_status step_expand_impl(etg_graph *g) {
     Launch ex;
     etg_status rc = expand_launch<OffT>(g, g->step_alg, ex);
     if (rc != ETG_OK) return rc;
-    uint32_t cap_e = g->p.ts * g->p.K;
+    uint32_t cap_e = expand_arg(g->p);
     void *exp_args[] = {&d, &cap_e};
-    if (g->p.warp) exp_args[1] = nullptr;
     ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, g->stream));
     g->step_launches += 1;
     return ETG_OK;
@@ -500,9 +512,8 @@ etg_status replay_impl(etg_graph *g, int alg, uint32_t source, uint32_t depth, u
     Launch ex;
     etg_status rc = expand_launch<OffT>(g, alg, ex);
     if (rc != ETG_OK) return rc;
-    uint32_t cap_e = g->p.ts * g->p.K;
+    uint32_t cap_e = expand_arg(g->p);
     void *exp_args[] = {&d, &cap_e};
-    if (g->p.warp) exp_args[1] = nullptr;
     cudaGraphConditionalHandle none = 0;
     int zero = 0;
     void *scan_args[] = {&d, &none, &zero};
@@ -526,7 +537,6 @@ etg_status replay_impl(etg_graph *g, int alg, uint32_t source, uint32_t depth, u
     Dev<OffT> dt = d;
     dt.tune = tune;
     void *targs[] = {&dt, &cap_e};
-    if (g->p.warp) targs[1] = nullptr;
     float total = 0.f;
     for (int r = 0; r < reps; ++r) {
         ETG_CU(cudaMemcpyAsync(label, saved, 4ull * g->n, cudaMemcpyDeviceToDevice, s));

@@ -90,24 +90,20 @@ struct Dev {
     unsigned long long *st_agg; //   aggregate  (entries << 32 | shadows)
     unsigned long long *st_inc; //   inclusive prefix, same packing
     Ctl *ctl;
+    unsigned long long m;       // edges
     uint32_t n;
     uint32_t nwords;            // bitmap words (padded to whole scan tiles)
     uint32_t K;                 // degree limit (Def. 3); unused with NO_UDC
     uint32_t ts;                // shadows per expand tile (<= kBlock, power of 2)
     uint32_t ts_log2;
     uint32_t tune;              // experiment switches (ETG_TUNE env var at load); 0 = default
+    uint32_t prefetch;          // warp kernel, direct mode: L2 bulk prefetch of the next tile
 };
 
 constexpr uint32_t kTuneFilterL1 = 1u;    // pre-filter label loads cached in L1
 // replay-only experiment switches (etg_debug_expand_replay; results not kept)
 constexpr uint32_t kTuneNoGather = 16u;   // skip the label gather and the commit
 constexpr uint32_t kTuneNoCommit = 32u;   // gather labels but never commit (counts passes)
-constexpr uint32_t kTuneBitOnly = 64u;    // commit = red.or of the bitmap only
-constexpr uint32_t kTuneNoPrefetch = 512u; // no L2 prefetch of the next tile's segments
-constexpr uint32_t kTuneStatic = 1024u;    // static round-robin tile schedule
-constexpr uint32_t kTuneRedMinOnly = 2048u; // commit: label reduction only (no bitmap mark)
-constexpr uint32_t kTuneRedOrOnly = 4096u;  // commit: bitmap mark only (no label reduction)
-constexpr uint32_t kTuneNoHint = 8192u;     // commit reductions without the L2 policy
 
 // ------------------------------------------------------------------------- //
 // small device helpers
@@ -714,9 +710,48 @@ __device__ __forceinline__ WarpShadow<OffT, UDC> warp_map(const Dev<OffT> &d, ui
     return r;
 }
 
-template <class OffT, int ALG, bool UDC>
-__global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT> d) {
+// ---- mbarrier / bulk-copy helpers (SMP stages) ----
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
+    asm volatile("{\n .reg .pred p;\n WAIT_%=:\n"
+                 " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+                 " @!p bra WAIT_%=;\n}" :: "r"(smem_u32(b)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+// TMA bulk copy global -> shared (16-byte aligned, size multiple of 16), completing on mbarrier b
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *b, uint64_t pol) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+                 :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(b)), "l"(pol) : "memory");
+}
+
+// Per-tile state of a warp: its 32 shadows and where their edges live.
+template <class OffT, bool UDC>
+struct WarpTile {
+    WarpShadow<OffT, UDC> sh;
+    uint32_t o;        // flat offset of this lane's slice in the tile
+    uint32_t E;        // edges in the tile
+    OffT delta;        // element x of this lane's slice is col[delta + x]      (direct)
+    uint32_t sdelta;   // ... and stage[sdelta + x] in shared memory            (SMP)
+};
+
+template <class OffT, int ALG, bool UDC, bool SMP>
+__global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT> d, uint32_t capw) {
     constexpr bool kW = (ALG == ALG_SSSP || ALG == ALG_SSWP);
+    constexpr uint32_t kArrays = kW ? 2u : 1u;
+    extern __shared__ __align__(128) uint8_t dyn_smem[];
     Ctl *ctl = d.ctl;
     const uint32_t nF = ctl->nF, N = ctl->nshadow, ntiles = ctl->ntiles;
     const uint32_t level = ctl->depth + 1;
@@ -724,7 +759,7 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
     uint32_t *Q = d.Q;
     const uint32_t lane = lane_id();
     const uint32_t lt_eq = (2u << lane) - 1u;
-    const bool l1 = (d.tune & kTuneFilterL1) != 0;
+    const uint32_t wib = threadIdx.x >> 5;                 // warp in block
     const uint64_t keep = policy_keep(), stream = policy_stream();
     unsigned long long my_edges = 0;
     uint32_t my_passes = 0;                               // replay experiment counter
@@ -736,21 +771,27 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
         ctl->frontier += nF;
         ctl->shadows += N;
     }
+    // SMP: two shared-memory stages per warp, each kArrays x capw words, and
+    // one mbarrier per stage (the TMA bulk copies complete on it).
+    uint32_t *wbuf = nullptr;
+    uint64_t *bars = nullptr;
+    if (SMP) {
+        wbuf = reinterpret_cast<uint32_t *>(dyn_smem) + (size_t)wib * 2u * kArrays * capw;
+        bars = reinterpret_cast<uint64_t *>(dyn_smem + (size_t)kWarps * 2u * kArrays * capw * 4u) + 2u * wib;
+        if (lane == 0) {
+            mbar_init(&bars[0], 1);
+            mbar_init(&bars[1], 1);
+            fence_mbar_init();
+        }
+        __syncwarp();
+    }
+    const OffT m_floor4 = (OffT)(d.m & ~3ull);            // whole 16-byte groups inside col/w
+
     // Dynamic schedule: a warp grabs kGrab consecutive tiles at a time, so the
     // slowest warp ends within one grab of the rest (tiles carry 32..32K edges).
-    // One-tile lookahead: the next tile is mapped, and its neighbour segments
-    // are prefetched into L2 (cp.async.bulk.prefetch), while the current tile is
-    // relaxed, so its column reads hit L2 instead of waiting on HBM.
     constexpr uint32_t kGrab = 2;
     uint32_t g_next = 0, g_end = 0;
-    const uint32_t gwarp = blockIdx.x * kWarps + (threadIdx.x >> 5), nwarps = gridDim.x * kWarps;
-    uint32_t s_next = gwarp;
     auto next_tile = [&]() -> uint32_t {
-        if (d.tune & kTuneStatic) {                       // static round-robin (experiment)
-            const uint32_t r = s_next;
-            s_next += nwarps;
-            return r < ntiles ? r : ntiles;
-        }
         if (g_next == g_end) {
             uint32_t g = 0;
             if (lane == 0) g = atomicAdd(&ctl->tile_ctr, kGrab);
@@ -760,120 +801,144 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
         }
         return g_next++;
     };
-    auto prefetch = [&](const WarpShadow<OffT, UDC> &w) {
-        if (w.len && !(d.tune & kTuneNoPrefetch)) {
-            const uintptr_t lo = reinterpret_cast<uintptr_t>(d.col + w.start) & ~(uintptr_t)15;
-            const uintptr_t hi = (reinterpret_cast<uintptr_t>(d.col + w.start + w.len) + 15) & ~(uintptr_t)15;
+    // Map tile t and start fetching its neighbour segments: SMP -> TMA bulk
+    // copies into stage `st` (Sec. V-B: fetch the shadow's neighbours to
+    // shared memory before processing them); direct -> L2 bulk prefetch.
+    auto prepare = [&](uint32_t t, uint32_t st) -> WarpTile<OffT, UDC> {
+        WarpTile<OffT, UDC> w;
+        w.sh = warp_map<OffT, UDC>(d, t, nF, N);
+        const uint32_t incl = warp_incl_scan(w.sh.len);
+        w.o = incl - w.sh.len;
+        w.E = __shfl_sync(kFull, incl, 31);
+        w.delta = w.sh.start - (OffT)w.o;
+        w.sdelta = 0;
+        if (SMP) {
+            // 16-byte-aligned superset of the slice (reading R-3: the over-fetched
+            // words are never relaxed); the tail past the last whole 16-byte
+            // group of col is loaded by the lane itself.
+            const OffT a_lo = w.sh.start & ~(OffT)3;
+            OffT a_hi = (w.sh.start + w.sh.len + 3) & ~(OffT)3;
+            const uint32_t pw = w.sh.len ? (uint32_t)(a_hi - a_lo) : 0u;
+            const uint32_t pincl = warp_incl_scan(pw);
+            const uint32_t slot = pincl - pw;
+            const uint32_t T = __shfl_sync(kFull, pincl, 31);
+            w.sdelta = slot + (uint32_t)(w.sh.start - a_lo) - w.o;
+            uint32_t *buf = wbuf + (size_t)st * kArrays * capw;
+            if (a_hi > m_floor4) a_hi = a_lo > m_floor4 ? a_lo : m_floor4;
+            const uint32_t tma_words = w.sh.len ? (uint32_t)(a_hi - a_lo) : 0u;
+            const uint32_t tma_total = __reduce_add_sync(kFull, tma_words);
+            if (lane == 0) mbar_expect_tx(&bars[st], tma_total * 4u * kArrays);
+            __syncwarp();
+            fence_proxy_async();
+            if (tma_words) {
+                bulk_g2s(buf + slot, d.col + a_lo, tma_words * 4u, &bars[st], stream);
+                if (kW) bulk_g2s(buf + capw + slot, d.w + a_lo, tma_words * 4u, &bars[st], stream);
+            }
+            // tail words [a_hi, start + len) (only the slice that ends the edge array)
+            for (OffT e = a_hi > w.sh.start ? a_hi : w.sh.start; e < w.sh.start + w.sh.len; ++e) {
+                buf[slot + (uint32_t)(e - a_lo)] = d.col[e];
+                if (kW) buf[capw + slot + (uint32_t)(e - a_lo)] = d.w[e];
+            }
+            (void)T;
+        } else if (w.sh.len && d.prefetch) {
+            const uintptr_t lo = reinterpret_cast<uintptr_t>(d.col + w.sh.start) & ~(uintptr_t)15;
+            const uintptr_t hi = (reinterpret_cast<uintptr_t>(d.col + w.sh.start + w.sh.len) + 15) & ~(uintptr_t)15;
             prefetch_l2(reinterpret_cast<const void *>(lo), (uint32_t)(hi - lo));
             if (kW) prefetch_l2(reinterpret_cast<const void *>(lo - reinterpret_cast<uintptr_t>(d.col) +
                                                                reinterpret_cast<uintptr_t>(d.w)),
                                 (uint32_t)(hi - lo));
         }
+        return w;
     };
+
     uint32_t t = next_tile();
-    if (t >= ntiles) {
-        if (lane == 0 && my_edges) atomicAdd(&ctl->edges, my_edges);
-        return;
-    }
-    WarpShadow<OffT, UDC> sh_next = warp_map<OffT, UDC>(d, t, nF, N);
-    prefetch(sh_next);
-    for (;;) {
-        const WarpShadow<OffT, UDC> sh = sh_next;
-        const uint32_t tn = next_tile();
-        if (tn < ntiles) {
-            sh_next = warp_map<OffT, UDC>(d, tn, nF, N);
-            prefetch(sh_next);
-        }
-        const uint32_t lab = (ALG == ALG_BFS) ? level
-                             : (sh.len ? ld_cg(&label[sh.v]) : 0u);   // fresh source label (R-6)
-        const uint32_t incl = warp_incl_scan(sh.len);
-        const uint32_t o = incl - sh.len;                     // flat offset of this lane's slice
-        const OffT delta = sh.start - (OffT)o;                // col index of element x = delta + x
-        const uint32_t E = __shfl_sync(kFull, incl, 31);
-        my_edges += E;
-        uint32_t owner = 0xFFFFFFFFu;                         // owner of the element before x0
-        // Batches of kR chunks of 32 elements.  The owner of element x is the
-        // number of slice starts <= x, minus one: the batch's kR words of the
-        // start mask come from kR independent OR-reductions, then a popcount
-        // prefix -- no serial dependency between the chunks of a batch.
-        for (uint32_t x0 = 0; x0 < E; x0 += 32u * kR) {
-            uint32_t u[kR], c[kR], cur[kR], wv[kR];
-            bool act[kR];
-            const uint32_t pos = o - x0;                      // this lane's slice start in the batch
-            const bool in_win = sh.len && pos < 32u * kR;
-            uint32_t wm[kR];
-#pragma unroll
-            for (int r = 0; r < kR; ++r)
-                wm[r] = __reduce_or_sync(kFull, (in_win && (pos >> 5) == (uint32_t)r) ? (1u << (pos & 31)) : 0u);
-#pragma unroll
-            for (int r = 0; r < kR; ++r) {
-                const uint32_t own = owner + __popc(wm[r] & lt_eq);
-                owner += __popc(wm[r]);
-                const uint32_t src = own & 31u;
-                const OffT dl = __shfl_sync(kFull, delta, src);
-                const uint32_t ll = (ALG == ALG_BFS) ? level : __shfl_sync(kFull, lab, src);
-                const uint32_t x = x0 + 32u * r + lane;
-                act[r] = x < E;
-                u[r] = 0;
-                c[r] = ll;
-                wv[r] = 0;
-                if (act[r]) {
-                    const OffT e = dl + (OffT)x;
-                    u[r] = ld_stream(&d.col[e], stream);
-                    if (kW) wv[r] = ld_stream(&d.w[e], stream);
-                }
+    if (t < ntiles) {
+        WarpTile<OffT, UDC> nxt = prepare(t, 0);
+        for (uint32_t k = 0;; ++k) {
+            const WarpTile<OffT, UDC> cur_t = nxt;
+            const uint32_t tn = next_tile();
+            if (tn < ntiles) nxt = prepare(tn, (k + 1) & 1);   // one tile ahead
+            const WarpShadow<OffT, UDC> &sh = cur_t.sh;
+            const uint32_t o = cur_t.o, E = cur_t.E;
+            const uint32_t lab = (ALG == ALG_BFS) ? level
+                                 : (sh.len ? ld_cg(&label[sh.v]) : 0u);   // fresh source label (R-6)
+            my_edges += E;
+            const uint32_t *sbuf = nullptr;
+            if (SMP) {
+                mbar_wait(&bars[k & 1], (k >> 1) & 1);
+                __syncwarp();
+                sbuf = wbuf + (size_t)(k & 1) * kArrays * capw;
             }
-            if (kW) {
-#pragma unroll
-                for (int r = 0; r < kR; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
-            }
-            if (d.tune & kTuneNoGather) {                     // replay experiment
-                uint32_t x = 0;
-#pragma unroll
-                for (int r = 0; r < kR; ++r) x += act[r] ? u[r] + c[r] : 0u;
-                if (x == 0x9E3779B9u) Q[0] = x;
-                continue;
-            }
-            // pre-filter: BFS reads the labels (written only by the scan); the
-            // others read the iteration-start snapshot, so the gathers and the
-            // red.min/max commits never touch the same lines (R-4, R-6)
-            const uint32_t *filt = (ALG == ALG_BFS) ? label : d.snap;
-#pragma unroll
-            for (int r = 0; r < kR; ++r)
-                cur[r] = act[r] ? (l1 ? ld_ca(&filt[u[r]]) : ld_label(&filt[u[r]], keep)) : 0u;
-            if (d.tune & kTuneNoCommit) {                     // replay experiment: count passes
-                uint32_t x = 0;
-#pragma unroll
-                for (int r = 0; r < kR; ++r) x += (act[r] && improves<ALG>(c[r], cur[r])) ? 1u : 0u;
-                my_passes += x;
-                continue;
-            }
-            if (d.tune & kTuneBitOnly) {                      // replay experiment: bitmap only
+            uint32_t owner = 0xFFFFFFFFu;                     // owner of the element before x0
+            // Batches of kR chunks of 32 elements.  The owner of element x is
+            // the number of slice starts <= x, minus one: the batch's kR words of
+            // the start mask come from kR independent OR-reductions, then a
+            // popcount prefix -- no serial dependency between chunks.
+            for (uint32_t x0 = 0; x0 < E; x0 += 32u * kR) {
+                uint32_t u[kR], c[kR], cur[kR], wv[kR];
+                bool act[kR];
+                const uint32_t pos = o - x0;                  // this lane's slice start in the batch
+                const bool in_win = sh.len && pos < 32u * kR;
+                uint32_t wm[kR];
 #pragma unroll
                 for (int r = 0; r < kR; ++r)
-                    if (act[r] && improves<ALG>(c[r], cur[r])) red_or(&Q[u[r] >> 5], 1u << (u[r] & 31), keep);
-                continue;
-            }
-            if (d.tune & (kTuneRedMinOnly | kTuneRedOrOnly | kTuneNoHint)) {   // replay experiments
+                    wm[r] = __reduce_or_sync(kFull, (in_win && (pos >> 5) == (uint32_t)r) ? (1u << (pos & 31)) : 0u);
 #pragma unroll
                 for (int r = 0; r < kR; ++r) {
-                    if (!(act[r] && improves<ALG>(c[r], cur[r]))) continue;
-                    if (d.tune & kTuneNoHint) {
-                        atomicMin(&label[u[r]], c[r]);
-                        atomicOr(&Q[u[r] >> 5], 1u << (u[r] & 31));
-                    } else if (d.tune & kTuneRedMinOnly) {
-                        red_min(&label[u[r]], c[r], keep);
+                    const uint32_t own = owner + __popc(wm[r] & lt_eq);
+                    owner += __popc(wm[r]);
+                    const uint32_t src = own & 31u;
+                    const uint32_t ll = (ALG == ALG_BFS) ? level : __shfl_sync(kFull, lab, src);
+                    const uint32_t x = x0 + 32u * r + lane;
+                    act[r] = x < E;
+                    u[r] = 0;
+                    c[r] = ll;
+                    wv[r] = 0;
+                    if (SMP) {
+                        const uint32_t sd = __shfl_sync(kFull, cur_t.sdelta, src);
+                        if (act[r]) {
+                            u[r] = sbuf[sd + x];
+                            if (kW) wv[r] = sbuf[capw + sd + x];
+                        }
                     } else {
-                        red_or(&Q[u[r] >> 5], 1u << (u[r] & 31), keep);
+                        const OffT dl = __shfl_sync(kFull, cur_t.delta, src);
+                        if (act[r]) {
+                            const OffT e = dl + (OffT)x;
+                            u[r] = ld_stream(&d.col[e], stream);
+                            if (kW) wv[r] = ld_stream(&d.w[e], stream);
+                        }
                     }
                 }
-                continue;
-            }
+                if (kW) {
 #pragma unroll
-            for (int r = 0; r < kR; ++r)
-                if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep);
+                    for (int r = 0; r < kR; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
+                }
+                if (d.tune & kTuneNoGather) {                 // replay experiment
+                    uint32_t x = 0;
+#pragma unroll
+                    for (int r = 0; r < kR; ++r) x += act[r] ? u[r] + c[r] : 0u;
+                    if (x == 0x9E3779B9u) Q[0] = x;
+                    continue;
+                }
+                // pre-filter: BFS reads the labels (written only by the scan);
+                // the others read the iteration-start snapshot, so the gathers
+                // and the red.min/max commits never touch the same lines (R-4, R-6)
+                const uint32_t *filt = (ALG == ALG_BFS) ? label : d.snap;
+#pragma unroll
+                for (int r = 0; r < kR; ++r) cur[r] = act[r] ? ld_label(&filt[u[r]], keep) : 0u;
+                if (d.tune & kTuneNoCommit) {                 // replay experiment: count passes
+                    uint32_t x = 0;
+#pragma unroll
+                    for (int r = 0; r < kR; ++r) x += (act[r] && improves<ALG>(c[r], cur[r])) ? 1u : 0u;
+                    my_passes += x;
+                    continue;
+                }
+#pragma unroll
+                for (int r = 0; r < kR; ++r)
+                    if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep);
+            }
+            if (tn >= ntiles) break;
         }
-        if (tn >= ntiles) break;
     }
     // statistics: one atomic per warp
     if (lane == 0 && my_edges) atomicAdd(&ctl->edges, my_edges);

@@ -118,11 +118,13 @@ def test_k_invariance(c1, c1sym, K):
     srcs = gg.sample_sources(c1, 2, K)
     check_all(c1, srcs, K=K)
     check_cc(c1sym, K=K)
+    if K <= 32:
+        check_all(c1, srcs[:1], K=K, flags=128)      # shared-memory SMP stages
 
 
-@pytest.mark.parametrize("flags", [2, 4, 32, 2 | 32, 4 | 32])
+@pytest.mark.parametrize("flags", [2, 4, 32, 2 | 32, 4 | 32, 128, 128 | 32])
 def test_flag_invariance(c1, c1sym, flags):
-    """UDC off (L88 baseline), SMP off (Fig. 6 ablation), host-driven loop."""
+    """UDC off (L88 baseline), SMP off (Fig. 6 ablation), shared-memory SMP, host-driven loop."""
     srcs = gg.sample_sources(c1, 2, 5)
     check_all(c1, srcs, flags=flags)
     check_cc(c1sym, flags=flags)
