@@ -163,6 +163,51 @@ def csr_from_keys(name: str, n: int, keys: torch.Tensor) -> Graph:
     return Graph(name, n, off, dst)
 
 
+_BUCKET_TUPLES = 1 << 27      # tuples per dedup bucket (tests lower it)
+
+
+class KeyBuckets:
+    """Accumulates (src, dst) tuples chunk by chunk, routed into source-range
+    buckets, so large graphs are deduplicated bucket by bucket (never one sort
+    of all tuples); concatenating the buckets in order keeps the CSR sorted."""
+
+    def __init__(self, n: int, total: int):
+        self.n = n
+        want = max(1, min(n, -(-total // _BUCKET_TUPLES)))      # buckets needed
+        self.shift = max(0, (max(n - 1, 1) // want).bit_length()) if want > 1 else 64
+        self.nb = 1 if want == 1 else ((n - 1) >> self.shift) + 1
+        self.parts = [[] for _ in range(self.nb)]
+
+    def add(self, src: torch.Tensor, dst: torch.Tensor) -> None:
+        keys = dedup_keys(src, dst, self.n)
+        if self.nb == 1:
+            self.parts[0].append(keys)
+            return
+        b = torch.div(keys, self.n, rounding_mode="floor") >> self.shift
+        bounds = torch.searchsorted(b, torch.arange(self.nb + 1, device=b.device))
+        for i in range(self.nb):
+            lo, hi = int(bounds[i]), int(bounds[i + 1])
+            if hi > lo:
+                self.parts[i].append(keys[lo:hi])
+
+    def csr(self, name: str, device) -> "Graph":
+        cnt = torch.zeros(self.n, dtype=torch.int64, device=device)
+        cols = []
+        for i in range(self.nb):
+            if not self.parts[i]:
+                continue
+            k = torch.unique(torch.cat(self.parts[i]), sorted=True)
+            self.parts[i] = None
+            src = torch.div(k, self.n, rounding_mode="floor")
+            cnt += torch.bincount(src, minlength=self.n)
+            cols.append(k - src * self.n)
+            del k, src
+        off = torch.zeros(self.n + 1, dtype=torch.int64, device=device)
+        off[1:] = torch.cumsum(cnt, 0)
+        col = torch.cat(cols) if cols else torch.zeros(0, dtype=torch.int64, device=device)
+        return Graph(name, self.n, off, col)
+
+
 def dedup_keys(src: torch.Tensor, dst: torch.Tensor, n: int) -> torch.Tensor:
     keep = src != dst                                     # drop self-loops
     keys = src[keep] * n + dst[keep]
@@ -230,7 +275,7 @@ def rmat(scale: int, edge_factor: int = 16, a: float = 0.45, b: float = 0.22,
     tABC = int(math.floor((a + b + c) * 2**32))
     key = seed_key(seed, 1)
     pkey = seed_key(seed, 2)
-    keys = []
+    acc = KeyBuckets(n, ntup)
     words = (scale + 1) // 2
     for lo in range(0, ntup, chunk):
         e = torch.arange(lo, min(ntup, lo + chunk), dtype=torch.int64, device=device)
@@ -251,10 +296,9 @@ def rmat(scale: int, edge_factor: int = 16, a: float = 0.45, b: float = 0.22,
         if permute:
             src = feistel_permute(src, n, pkey)
             dst = feistel_permute(dst, n, pkey)
-        keys.append(dedup_keys(src, dst, n))
+        acc.add(src, dst)
         del e, src, dst
-    allk = torch.unique(torch.cat(keys), sorted=True) if len(keys) > 1 else keys[0]
-    return csr_from_keys(name or f"rmat{scale}", n, allk)
+    return acc.csr(name or f"rmat{scale}", device)
 
 
 # --------------------------------------------------------------------------- #
@@ -290,7 +334,7 @@ def chung_lu(n: int, m_target: int, alpha_out: float, dmax_out: float,
         cum.append(torch.from_numpy(np.cumsum(q)).to(device))
     key_s, key_d = seed_key(seed, 3), seed_key(seed, 4)
     perm_s, perm_d = seed_key(seed, 5), seed_key(seed, 6)
-    keys = []
+    acc = KeyBuckets(n, ntup)
     for lo in range(0, ntup, chunk):
         e = torch.arange(lo, min(ntup, lo + chunk), dtype=torch.int64, device=device)
         ends = []
@@ -298,10 +342,9 @@ def chung_lu(n: int, m_target: int, alpha_out: float, dmax_out: float,
             t = torch.remainder(_srl(rand64(k, e), 1), int(cw[-1]))
             idx = torch.searchsorted(cw, t, right=True)
             ends.append(feistel_permute(idx, n, pk))
-        keys.append(dedup_keys(ends[0], ends[1], n))
+        acc.add(ends[0], ends[1])
         del e, ends
-    allk = torch.unique(torch.cat(keys), sorted=True) if len(keys) > 1 else keys[0]
-    return csr_from_keys(name, n, allk)
+    return acc.csr(name, device)
 
 
 # --------------------------------------------------------------------------- #

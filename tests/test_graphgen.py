@@ -78,3 +78,15 @@ def test_symmetrize():
     off, col, _ = s.numpy()
     assert off.tolist() == [0, 1, 3, 4, 4]
     assert col.tolist() == [1, 0, 2, 1]
+
+
+def test_bucketed_dedup_is_equivalent(monkeypatch):
+    """Large graphs are deduplicated per source-range bucket: same CSR."""
+    a = gg.make("T12")
+    monkeypatch.setattr(gg, "_BUCKET_TUPLES", 1 << 10)
+    b = gg.make("T12")
+    assert a.sha256() == b.sha256()
+    c = gg.make("LJ-small", weights=False)
+    monkeypatch.setattr(gg, "_BUCKET_TUPLES", 1 << 27)
+    d = gg.make("LJ-small", weights=False)
+    assert c.sha256() == d.sha256()
