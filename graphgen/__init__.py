@@ -360,7 +360,7 @@ CONFIGS = {
                dmax_out=20_000, alpha_in=2.0, dmax_in=14_000, oversample=1.03, seed=3),
     # C4: Twitter-shaped Chung-Lu (41.6M vertices, ~1.47B edges)
     "C4": dict(kind="chunglu", n=41_600_000, m_target=1_470_000_000, alpha_out=1.7,
-               dmax_out=3_000_000, alpha_in=2.1, dmax_in=300_000, oversample=1.16, seed=41),
+               dmax_out=3_000_000, alpha_in=2.1, dmax_in=300_000, oversample=1.33, seed=41),
     # C5: RMAT scale-28 (268M vertices, 4.3B tuples)
     "C5": dict(kind="rmat", scale=28, edge_factor=16, seed=28),
     # small variants used by tests
