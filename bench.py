@@ -59,6 +59,9 @@ def parse_args():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-profile", action="store_true")
     p.add_argument("--json-out", default=None)
+    p.add_argument("--partitioned", action="store_true",
+                   help="1-D destination partition of ONE graph over the N ranks (NCCL exchange); "
+                        "default: N independent replicas")
     return p.parse_args()
 
 
@@ -507,10 +510,88 @@ def run_ours(args):
     return 0
 
 
+def run_partitioned(args):
+    """One graph split over the N ranks: every rank expands the
+    replicated active set over its destination partition; NCCL all-reduce
+    exchange per iteration.  Strong scaling: the same traversals at every N."""
+    import torch
+    import torch.distributed as tdist
+    import graphgen as gg
+    import paper_conf_ipps_wangzlg19_b200 as etg
+    from paper_conf_ipps_wangzlg19_b200 import _build, dist as edist
+
+    rank, world, local = dist_setup()
+    if rank == 0:
+        _build.build()
+    barrier(world)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    algs = args.algs.split(",")
+    alg_id = {"bfs": etg.BFS, "sssp": etg.SSSP, "cc": etg.CC}
+    res = {}
+    for a in algs:
+        g = gg.make(args.config, device=dev, weights=(a == "sssp"), symmetric=(a == "cc"))
+        deg = g.degrees()
+        sources = gg.sample_sources(g, args.sources, 4242)           # the same on every rank
+        group = None
+        if world == 1:
+            import torch.distributed as d0
+            if not d0.is_initialized():
+                d0.init_process_group("nccl", init_method="tcp://127.0.0.1:29555", rank=0, world_size=1,
+                                      device_id=dev)
+        dg = edist.DistGraph(g.off, g.col, g.w, g.n, rank, world, K=args.K, flags=args.flags,
+                             symmetric=(a == "cc"), device=dev, group=group)
+        m_sym = g.m
+        del g
+        torch.cuda.empty_cache()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ms_tot, edges_tot = 0.0, 0
+        for i in range(args.warmup + args.steps):
+            s = sources[i % len(sources)]
+            barrier(world)
+            torch.cuda.synchronize()
+            ev0.record()
+            labels, st = dg.run(alg_id[a], s)
+            ev1.record()
+            torch.cuda.synchronize()
+            if i >= args.warmup:
+                ms_tot += ev0.elapsed_time(ev1)
+                unreached = etg.INF
+                reached = labels.view(torch.int32) != -1 if a != "cc" else None
+                edges_tot += m_sym if a == "cc" else int(deg[reached].sum())
+        ms_max = allreduce([ms_tot], tdist.ReduceOp.MAX, world)[0] if world > 1 else ms_tot
+        res[a] = {"gteps": edges_tot / ms_max / 1e6, "ms_per_call": ms_max / args.steps, "edges": edges_tot,
+                  "ms": ms_max}
+        del dg, deg
+        torch.cuda.empty_cache()
+    tot_e = sum(v["edges"] for v in res.values())
+    tot_ms = sum(v["ms"] for v in res.values())
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": tot_e / tot_ms / 1e6, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_ms / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": config_desc(args.config) + "; " + "+".join(algs) + " per step",
+                       "parallelism": f"1-D destination partition over {world} GPU(s), NCCL all-reduce exchange",
+                       "K": args.K, "flags": args.flags},
+            "per_alg": {k: {"gteps": v["gteps"], "ms_per_call": v["ms_per_call"]} for k, v in res.items()},
+        }
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.json_out:
+            with open(args.json_out, "w") as f:
+                f.write(s + "\n")
+    if torch.distributed.is_initialized():
+        torch.distributed.destroy_process_group()
+    return 0
+
+
 def main():
     args = parse_args()
     if args.impl == "reference":
         return run_reference(args)
+    if args.partitioned:
+        return run_partitioned(args)
     return run_ours(args)
 
 

@@ -15,8 +15,9 @@ Design:
   non-owner's copy is the owner's value from an earlier exchange, never better
   than the owner's current one.  BFS exchanges the bitmap only -- each rank's
   scan writes the depth of every vertex of the new active set.
-* termination: the compacted active-set size after the exchange is identical
-  on every rank (same bitmap), so all ranks leave the loop together.
+* termination: the number of activated vertices (bitmap bits consumed by the
+  scan) is identical on every rank after the exchange, so all ranks leave the
+  loop together (the compacted sizes differ: they count local out-edges).
 
 Only argument marshalling and the collective calls are in Python; every step of
 the traversal runs in libetg.so (etg_step_begin / etg_step_expand /
@@ -59,18 +60,30 @@ def partition_ranges(off: torch.Tensor, col: torch.Tensor, n: int, P: int, align
 
 
 def partition_csr(off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor], n: int,
-                  lo: int, hi: int):
+                  lo: int, hi: int, chunk: int = 1 << 28):
     """The rank's destination-partitioned CSR: rows = all n sources, edges with
-    destination in [lo, hi), CSR order kept, global ids."""
+    destination in [lo, hi), CSR order kept, global ids.  Processed in edge
+    chunks (no m-sized int64 temporaries), kept columns stored as int32 bits."""
     off = off.to(torch.int64)
-    col = col.to(torch.int64)
-    keep = (col >= lo) & (col < hi)
-    src = torch.repeat_interleave(torch.arange(n, device=off.device), off[1:] - off[:-1])
-    src = src[keep]
-    cnt = torch.bincount(src, minlength=n)
-    loff = torch.zeros(n + 1, dtype=torch.int64, device=off.device)
+    m = int(col.shape[0])
+    dev = off.device
+    cnt = torch.zeros(n, dtype=torch.int64, device=dev)
+    cols, ws = [], []
+    for a in range(0, m, chunk):
+        b = min(m, a + chunk)
+        c = col[a:b].to(torch.int64)
+        keep = (c >= lo) & (c < hi)
+        src = torch.searchsorted(off, torch.arange(a, b, device=dev), right=True) - 1
+        cnt += torch.bincount(src[keep], minlength=n)
+        cols.append(c[keep].to(torch.int32))
+        if w is not None:
+            ws.append(w[a:b][keep].to(torch.int32))
+        del c, keep, src
+    loff = torch.zeros(n + 1, dtype=torch.int64, device=dev)
     loff[1:] = torch.cumsum(cnt, 0)
-    return loff, col[keep], (None if w is None else w.to(torch.int64)[keep])
+    lcol = torch.cat(cols) if cols else torch.zeros(0, dtype=torch.int32, device=dev)
+    lw = (torch.cat(ws) if ws else torch.zeros(0, dtype=torch.int32, device=dev)) if w is not None else None
+    return loff, lcol, lw
 
 
 # --------------------------------------------------------------------------- #
