@@ -536,8 +536,11 @@ def run_partitioned(args):
         if world == 1:
             import torch.distributed as d0
             if not d0.is_initialized():
-                d0.init_process_group("nccl", init_method="tcp://127.0.0.1:29555", rank=0, world_size=1,
-                                      device_id=dev)
+                if "MASTER_ADDR" in os.environ:          # under torchrun: its env:// rendezvous
+                    d0.init_process_group("nccl", device_id=dev)
+                else:
+                    d0.init_process_group("nccl", init_method="tcp://127.0.0.1:29555", rank=0,
+                                          world_size=1, device_id=dev)
         dg = edist.DistGraph(g.off, g.col, g.w, g.n, rank, world, K=args.K, flags=args.flags,
                              symmetric=(a == "cc"), device=dev, group=group)
         m_sym = g.m
