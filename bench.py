@@ -53,6 +53,7 @@ def parse_args():
     p.add_argument("--config", default="C2")
     p.add_argument("--algs", default="bfs,sssp,cc")
     p.add_argument("--K", type=int, default=32)
+    p.add_argument("--sssp-delta", type=int, default=0, help="near-far SSSP bucket width (0: paper schedule)")
     p.add_argument("--flags", type=int, default=0, help="extra ETG_* flags (e.g. 2 = NO_UDC)")
     p.add_argument("--sources", type=int, default=16)
     p.add_argument("--no-e2e", action="store_true")
@@ -323,7 +324,8 @@ def run_ours(args):
 
     def mk(graph, flags, sym=False):
         o, c, w, fl = etg.csr_to_device(graph.off, graph.col, graph.w, device=dev)
-        return etg.Graph(o, c, w, n=graph.n, K=args.K, flags=flags | fl | args.flags, symmetric=sym)
+        return etg.Graph(o, c, w, n=graph.n, K=args.K, flags=flags | fl | args.flags, symmetric=sym,
+                         sssp_delta=args.sssp_delta)
 
     G = mk(g, 0)
     Gs = mk(gs, 0, sym=True) if gs is not None else None

@@ -76,6 +76,12 @@ enum {
 typedef struct {
     uint32_t degree_limit_k; /* K of Def. 3; 0 -> default 32 */
     uint32_t flags;          /* ETG_* bits above */
+    uint32_t sssp_delta;     /* 0: the paper's schedule (every improved vertex is active in the
+                                next iteration, L64/L78).  > 0: near-far schedule for SSSP --
+                                improved vertices at distance >= a threshold stay active but are
+                                deferred; the threshold advances by sssp_delta when no nearer
+                                vertex is active.  Same distances (unique fixpoint), fewer
+                                redundant relaxations.  Ignored by the step-wise (multi-GPU) API. */
 } etg_options;
 
 typedef struct {

@@ -41,7 +41,8 @@ class EtgError(RuntimeError):
 
 
 class Options(ctypes.Structure):
-    _fields_ = [("degree_limit_k", ctypes.c_uint32), ("flags", ctypes.c_uint32)]
+    _fields_ = [("degree_limit_k", ctypes.c_uint32), ("flags", ctypes.c_uint32),
+                ("sssp_delta", ctypes.c_uint32)]
 
 
 class Stats(ctypes.Structure):
@@ -154,7 +155,7 @@ class Graph:
 
     def __init__(self, off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor] = None, *,
                  n: Optional[int] = None, K: int = 32, flags: int = 0, symmetric: bool = False,
-                 validate: bool = False, stream=None):
+                 validate: bool = False, stream=None, sssp_delta: int = 0):
         if not torch.cuda.is_available():
             raise EtgError("no CUDA device: etg has no CPU fallback")
         if off.dtype == torch.int64:
@@ -177,7 +178,7 @@ class Graph:
         self.device = off.device
         self._keep = (off, col, w)
         self._stream = stream
-        self._opt = Options(K, flags)
+        self._opt = Options(K, flags, sssp_delta)
         L = lib()
         nbytes = L.etg_workspace_bytes(self.n, self.m, ctypes.byref(self._opt))
         self.workspace = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=self.device)
@@ -284,13 +285,13 @@ def load_csr(off, col, w=None, **kw) -> Graph:
 
 
 def host_scratch_bytes(n: int, m: int, has_weights: bool, K: int = 32, flags: int = 0) -> int:
-    opt = Options(K, flags)
+    opt = Options(K, flags, 0)
     return int(lib().etg_host_scratch_bytes(n, m, int(has_weights), ctypes.byref(opt)))
 
 
 def run_host(alg: int, off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor],
              source: int, labels_out: torch.Tensor, scratch: torch.Tensor, *, K: int = 32,
-             flags: int = 0, stream=None) -> Stats:
+             flags: int = 0, stream=None, sssp_delta: int = 0) -> Stats:
     """End-to-end call on HOST tensors (pinned recommended): H2D, traverse, D2H."""
     for t in (off, col, w, labels_out):
         if t is not None and t.is_cuda:
@@ -301,7 +302,7 @@ def run_host(alg: int, off: torch.Tensor, col: torch.Tensor, w: Optional[torch.T
         flags |= SYMMETRIC
     n = int(off.shape[0] - 1)
     m = int(col.shape[0])
-    opt = Options(K, flags)
+    opt = Options(K, flags, sssp_delta)
     st = Stats()
     rc = lib().etg_run_host(alg, n, m, _ptr(off), _ptr(col), _ptr(w), source, _ptr(labels_out),
                             _ptr(scratch), scratch.numel() * scratch.element_size(),

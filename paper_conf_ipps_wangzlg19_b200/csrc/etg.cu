@@ -57,11 +57,13 @@ struct Params {
     bool smp;
     bool prefetch;  // warp kernel: L2 bulk prefetch of the next tile's segments
     bool u64;
+    uint32_t nf_delta;  // near-far SSSP bucket width (0 = paper schedule)
 };
 
 Params derive(const etg_options *opt, uint32_t tune) {
     Params p;
     p.warp = !(tune & 2u);
+    p.nf_delta = opt ? opt->sssp_delta : 0u;
     const uint32_t flags = opt ? opt->flags : 0u;
     p.K = (opt && opt->degree_limit_k) ? opt->degree_limit_k : 32u;
     p.udc = !(flags & ETG_NO_UDC);
@@ -154,8 +156,9 @@ struct etg_graph {
 namespace {
 
 template <class OffT>
-Dev<OffT> make_dev(const etg_graph *g) {
+Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     Dev<OffT> d;
+    d.nf_delta = (alg == ALG_SSSP) ? g->p.nf_delta : 0u;
     d.off = static_cast<const OffT *>(g->off);
     d.col = g->col;
     d.w = g->w;
@@ -267,7 +270,7 @@ etg_status expand_launch(etg_graph *g, int alg, Launch &out) {
 template <class OffT>
 etg_status build_graph(etg_graph *g, int alg) {
     if (g->exec[alg]) return ETG_OK;
-    Dev<OffT> d = make_dev<OffT>(g);
+    Dev<OffT> d = make_dev<OffT>(g, alg);
     Launch ex;
     etg_status s = expand_launch<OffT>(g, alg, ex);
     if (s != ETG_OK) return s;
@@ -312,7 +315,7 @@ etg_status build_graph(etg_graph *g, int alg) {
 
 template <class OffT>
 etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stats *st) {
-    Dev<OffT> d = make_dev<OffT>(g);
+    Dev<OffT> d = make_dev<OffT>(g, alg);
     cudaStream_t s = g->stream;
     const bool profile = (g->flags & ETG_PROFILE) != 0;
     const bool host_loop = profile || (g->flags & ETG_HOST_LOOP) != 0;
@@ -324,6 +327,7 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
     }
     ETG_CU(cudaEventRecord(g->ev0, s));
     ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, label, source);
+    if (d.nf_delta) ctl_nearfar_kernel<<<1, 1, 0, s>>>(g->ctl, d.nf_delta);
     {
         void *args[] = {&d, &label, &source};
         ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), args, 0, s));
@@ -342,9 +346,9 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
         void *exp_args[] = {&d, &cap_e};
             for (;;) {
             // "while actSet.isNotEmpty()" (L207): read the compacted size back
-            ETG_CU(cudaMemcpyAsync(&g->h_ctl->nF, &g->ctl->nF, 4, cudaMemcpyDeviceToHost, s));
+            ETG_CU(cudaMemcpyAsync(&g->h_ctl->more, &g->ctl->more, 4, cudaMemcpyDeviceToHost, s));
             ETG_CU(cudaStreamSynchronize(s));
-            if (g->h_ctl->nF == 0) break;
+            if (g->h_ctl->more == 0) break;
             if (profile) ETG_CU(cudaEventRecord(g->pev[0], s));
             ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
             if (profile) ETG_CU(cudaEventRecord(g->pev[1], s));

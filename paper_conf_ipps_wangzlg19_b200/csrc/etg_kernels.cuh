@@ -71,7 +71,10 @@ struct Ctl {
     unsigned long long reached_e;
     uint32_t *label;      // output label array of the current call
     uint32_t source;
-    uint32_t pad;
+    uint32_t thresh;      // near-far SSSP: marked vertices with label < thresh are expanded
+    uint32_t far_min;     //   min label of the deferred (far) marked vertices of the last scan
+    uint32_t far_count;   //   number of deferred marked vertices of the last scan
+    uint32_t more;        // loop condition computed by the last scan
 };
 
 template <class OffT>
@@ -98,6 +101,7 @@ struct Dev {
     uint32_t ts_log2;
     uint32_t tune;              // experiment switches (ETG_TUNE env var at load); 0 = default
     uint32_t prefetch;          // warp kernel, direct mode: L2 bulk prefetch of the next tile
+    uint32_t nf_delta;          // near-far SSSP bucket width (0: the paper's schedule)
 };
 
 constexpr uint32_t kTuneFilterL1 = 1u;    // pre-filter label loads cached in L1
@@ -211,12 +215,14 @@ __device__ __forceinline__ T block_excl_scan(T x, T *wsum, T &total) {
     T incl = warp_incl_scan(x);
     const uint32_t warp = threadIdx.x >> 5;
     if (lane_id() == 31) wsum[warp] = incl;
+    __syncwarp();                                   // bar.sync needs converged warps
     __syncthreads();
     if (warp == 0) {
         T s = lane_id() < (uint32_t)kWarps ? wsum[lane_id()] : T(0);
         s = warp_incl_scan(s);
         if (lane_id() < (uint32_t)kWarps) wsum[lane_id()] = s;
     }
+    __syncwarp();
     __syncthreads();
     T warp_prefix = warp ? wsum[warp - 1] : T(0);
     total = wsum[kWarps - 1];
@@ -250,7 +256,13 @@ __global__ void ctl_begin_kernel(Ctl *ctl, uint32_t *label, uint32_t source) {
     ctl->frontier = 0;
     ctl->label = label;
     ctl->source = source;
+    ctl->thresh = 0xFFFFFFFFu;
+    ctl->far_min = 0xFFFFFFFFu;
+    ctl->far_count = 0;
 }
+
+// near-far SSSP: the first threshold (the source has distance 0)
+__global__ void ctl_nearfar_kernel(Ctl *ctl, uint32_t delta) { ctl->thresh = delta; }
 
 // BFS/SSSP: label = INF, label[s] = 0, Q = {s}.  SSWP: label = 0, label[s] =
 // INF, Q = {s}.  CC: label[v] = v, Q = all vertices (the scan drops degree-0
@@ -334,13 +346,40 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
     const uint32_t new_depth = ctl->depth + 1;      // BFS depth of the vertices in Q
     for (;;) {
         if (threadIdx.x == 0) s_tile = atomicAdd(&ctl->scan_ctr, 1u);
+        __syncwarp();
         __syncthreads();
         const uint32_t tile = s_tile;
+        __syncthreads();                                  // all have read s_tile before it is reused
         if (tile >= nscan) break;
         const uint32_t v0 = tile * kScanV + threadIdx.x * kVT;
         // this thread's bitmap word (read and cleared)
-        const uint32_t bits = v0 < n ? d.Q[v0 >> 5] : 0u;
-        if (bits) d.Q[v0 >> 5] = 0u;
+        uint32_t bits = v0 < n ? d.Q[v0 >> 5] : 0u;
+        uint32_t far_bits = 0, far_min = kInf;
+        if (bits && d.nf_delta) {
+            // near-far SSSP: marked vertices at distance >= thresh stay marked
+            // (deferred, still active) and are not expanded in this iteration
+            const uint32_t th = ctl->thresh;
+            for (uint32_t b = bits; b; b &= b - 1) {
+                const uint32_t k = __ffs(b) - 1;
+                const uint32_t lv = __ldcg(&label[v0 + k]);
+                d.snap[v0 + k] = lv;                          // refresh the pre-filter snapshot
+                if (lv >= th) {
+                    far_bits |= 1u << k;
+                    far_min = min(far_min, lv);
+                }
+            }
+            bits &= ~far_bits;
+        }
+        if (bits | far_bits) d.Q[v0 >> 5] = far_bits;
+        if (d.nf_delta) {
+            const uint32_t fc = __reduce_add_sync(kFull, (uint32_t)__popc(far_bits));
+            const uint32_t fm = __reduce_min_sync(kFull, far_min);
+            if (lane == 0 && fc) {
+                atomicAdd(&ctl->far_count, fc);
+                atomicMin(&ctl->far_min, fm);
+            }
+            __threadfence();                                  // before this tile publishes
+        }
         OffT o[kVT + 1];
         u64 tsum = 0;
         if (bits) {
@@ -395,6 +434,7 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
                 }
             }
             if (lane == 0) s_prefix = excl;
+            __syncwarp();
         }
         __syncthreads();
         // pass 2: write the compacted entries (offsets still in registers)
@@ -405,7 +445,7 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
                 if (bits & (1u << k)) {
                     const uint32_t v = v0 + k;
                     if (BFSLAB) label[v] = new_depth;      // BFS: depth written once, on compaction
-                    else if (label) d.snap[v] = __ldcg(&label[v]);   // refresh the pre-filter snapshot
+                    else if (label && !d.nf_delta) d.snap[v] = __ldcg(&label[v]);   // refresh the snapshot
                     const uint32_t dg = (uint32_t)(o[k + 1] - o[k]);
                     const uint32_t c = udc_count<UDC>(dg, d.K);
                     if (c) {
@@ -434,8 +474,18 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
             ctl->ntiles = (N + ts - 1) >> tsl;
             ctl->tile_ctr = 0;
             ctl->depth += 1;
-            if (use_cond) cudaGraphSetConditional(cond, nF > 0 ? 1u : 0u);
+            bool more = nF > 0;
+            if (d.nf_delta && ctl->far_count) {
+                more = true;
+                if (nF == 0) {                        // near set empty: next bucket
+                    const unsigned long long th = (unsigned long long)ctl->far_min + d.nf_delta;
+                    ctl->thresh = th > kInf ? kInf : (uint32_t)th;
+                }
+            }
+            ctl->more = more ? 1u : 0u;
+            if (use_cond) cudaGraphSetConditional(cond, more ? 1u : 0u);
         }
+        __syncwarp();
         __syncthreads();
     }
 }
@@ -559,6 +609,8 @@ __global__ __launch_bounds__(kBlock) void expand_kernel(Dev<OffT> d, uint32_t ca
     if (blockIdx.x == 0 && tid == 0) {
         // bookkeeping for the scan that follows this kernel (stream-ordered)
         ctl->scan_ctr = 0;
+        ctl->far_min = kInf;
+        ctl->far_count = 0;
         ctl->epoch += 1;
         if (nF) ctl->iterations += 1;
         ctl->frontier += nF;
@@ -767,6 +819,8 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
         // bookkeeping for the scan that follows this kernel (stream-ordered)
         ctl->scan_ctr = 0;
         ctl->epoch += 1;
+        ctl->far_min = kInf;
+        ctl->far_count = 0;
         if (nF) ctl->iterations += 1;
         ctl->frontier += nF;
         ctl->shadows += N;
@@ -841,12 +895,16 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
             }
             (void)T;
         } else if (w.sh.len && d.prefetch) {
+            // whole 16-byte groups inside col only (never past the array's end)
             const uintptr_t lo = reinterpret_cast<uintptr_t>(d.col + w.sh.start) & ~(uintptr_t)15;
-            const uintptr_t hi = (reinterpret_cast<uintptr_t>(d.col + w.sh.start + w.sh.len) + 15) & ~(uintptr_t)15;
-            prefetch_l2(reinterpret_cast<const void *>(lo), (uint32_t)(hi - lo));
-            if (kW) prefetch_l2(reinterpret_cast<const void *>(lo - reinterpret_cast<uintptr_t>(d.col) +
-                                                               reinterpret_cast<uintptr_t>(d.w)),
-                                (uint32_t)(hi - lo));
+            uintptr_t hi = (reinterpret_cast<uintptr_t>(d.col + w.sh.start + w.sh.len) + 15) & ~(uintptr_t)15;
+            const uintptr_t end = reinterpret_cast<uintptr_t>(d.col + m_floor4);
+            if (hi > end) hi = end;
+            if (hi > lo) prefetch_l2(reinterpret_cast<const void *>(lo), (uint32_t)(hi - lo));
+            if (kW && hi > lo)
+                prefetch_l2(reinterpret_cast<const void *>(lo - reinterpret_cast<uintptr_t>(d.col) +
+                                                           reinterpret_cast<uintptr_t>(d.w)),
+                            (uint32_t)(hi - lo));
         }
         return w;
     };

@@ -10,7 +10,7 @@ def load_golden(name):
         return json.load(f)
 
 
-def to_etg(g, K=32, flags=0, symmetric=None, device="cuda", force_u64=False):
+def to_etg(g, K=32, flags=0, symmetric=None, device="cuda", force_u64=False, sssp_delta=0):
     """graphgen.Graph -> paper_conf_ipps_wangzlg19_b200.Graph on the device."""
     import torch
     import paper_conf_ipps_wangzlg19_b200 as etg
@@ -18,7 +18,8 @@ def to_etg(g, K=32, flags=0, symmetric=None, device="cuda", force_u64=False):
     if force_u64:
         o = g.off.to(device=device, dtype=torch.int64).contiguous()
     sym = g.symmetric if symmetric is None else symmetric
-    return etg.Graph(o, c, w, n=g.n, K=K, flags=flags | fl, symmetric=sym, validate=True)
+    return etg.Graph(o, c, w, n=g.n, K=K, flags=flags | fl, symmetric=sym, validate=True,
+                     sssp_delta=sssp_delta)
 
 
 def sssp_certificate_gpu(g, s, dist, chunk=1 << 27):

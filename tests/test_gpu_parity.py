@@ -266,3 +266,25 @@ def test_errors():
     bad = gg.Graph("bad", 3, torch.tensor([0, 1, 1, 1]), torch.tensor([7]))
     with pytest.raises(etg.EtgError, match="EINVALID_CSR"):
         to_etg(bad)
+
+
+@pytest.mark.parametrize("delta", [1, 7, 16, 64, 1 << 20])
+def test_sssp_near_far_schedule(c1, delta):
+    """The near-far schedule defers far active vertices; distances are the same
+    unique fixpoint (golden F2, saturation, C1, LJ-small, hub)."""
+    off, col, w = c1.numpy()
+    for s in gg.sample_sources(c1, 3, delta):
+        G = to_etg(c1, sssp_delta=delta)
+        np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
+        Gh = to_etg(c1, sssp_delta=delta, flags=32)
+        np.testing.assert_array_equal(U32(Gh.sssp(s)[0]), oracle.sssp(off, col, w, s))
+    f = load_golden("F2_sssp_reactivation.json")
+    G = to_etg(_fixture_graph(f), sssp_delta=delta)
+    assert U32(G.sssp(f["source"])[0]).tolist() == f["expect_sssp"]
+    f = load_golden("F4_saturation.json")
+    G = to_etg(_fixture_graph(f), sssp_delta=delta)
+    assert U32(G.sssp(f["source"])[0]).tolist() == f["expect_sssp"]
+    g = gg.make("LJ-small")
+    off, col, w = g.numpy()
+    s = gg.first_source(g)
+    np.testing.assert_array_equal(U32(to_etg(g, sssp_delta=delta).sssp(s)[0]), oracle.sssp(off, col, w, s))

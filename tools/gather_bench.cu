@@ -76,6 +76,11 @@ int main(int argc, char **argv) {
         cudaMemcpy(idx, h, got * 4, cudaMemcpyHostToDevice);
         free(h);
     }
+    for (int bps : {1, 2}) {
+        run<8, 0>("ld.cg", idx, lab, n_idx, out, sms, bps, 256);
+        run<16, 0>("ld.cg", idx, lab, n_idx, out, sms, bps, 256);
+        run<32, 0>("ld.cg", idx, lab, n_idx, out, sms, bps, 256);
+    }
     for (int bps : {4, 8}) {
         run<1, 0>("ld.cg", idx, lab, n_idx, out, sms, bps, 256);
         run<8, 0>("ld.cg", idx, lab, n_idx, out, sms, bps, 256);
