@@ -291,43 +291,19 @@ __global__ __launch_bounds__(kBlock) void init_kernel(Dev<OffT> d, uint32_t *lab
 
 // ------------------------------------------------------------------------- //
 // A5/A6 + A2 of the next iteration: bitmap -> compacted active set + UDC scan.
-// Scan tile = kScanV vertices; thread tid owns the kVT consecutive vertices
-// v0 = tile*kScanV + tid*kVT .. v0+kVT-1: their kVT bits of Q and, when any is
-// set, the kVT+1 row offsets off[v0 .. v0+kVT] read with vector loads
-// (coalesced across the warp), from which every degree follows -- no per-
-// vertex gather and no second gather in pass 2.  Persistent CTAs take scan
-// tiles in order from a counter, so the look-back always makes progress.
-// Values are packed (kept entries << 32 | shadows); neither half can carry
-// into the other (entries <= n < 2^32, shadows < 2^32 checked at load time).
-// The look-back is warp-parallel (32 predecessors per step).
+// Scan tile = kScanV vertices; warp w of the CTA owns kWPW consecutive bitmap
+// words, and lane l handles bit l of each: for word k the warp looks at the
+// 32 consecutive vertices 32k .. 32k+31, so the off[] loads, the label
+// writes and the compacted F/B/D/S stores are all coalesced; positions come
+// from a ballot/popcount (kept entries) and a warp scan (shadow counts).
+// Persistent CTAs take scan tiles in order from a counter, so the chained
+// (decoupled look-back) scan always makes progress.  Values are packed
+// (kept entries << 32 | shadows); neither half can carry into the other
+// (entries <= n < 2^32, shadows < 2^32 checked at load time).
 // ------------------------------------------------------------------------- //
-constexpr int kVT = 32;                          // vertices per thread (one bitmap word)
-constexpr uint32_t kScanV = kBlock * kVT;        // vertices per scan tile (8192 = 256 words)
-
-template <class OffT>
-__device__ __forceinline__ void load_offsets(const OffT *off, uint32_t v0, uint32_t n, OffT (&o)[kVT + 1]) {
-    if (v0 + kVT <= n) {
-        if (sizeof(OffT) == 4) {
-            const uint4 *p = reinterpret_cast<const uint4 *>(off + v0);
-#pragma unroll
-            for (int k = 0; k < kVT / 4; ++k) {
-                const uint4 q = __ldg(p + k);
-                o[4 * k] = (OffT)q.x; o[4 * k + 1] = (OffT)q.y; o[4 * k + 2] = (OffT)q.z; o[4 * k + 3] = (OffT)q.w;
-            }
-        } else {
-            const ulonglong2 *p = reinterpret_cast<const ulonglong2 *>(off + v0);
-#pragma unroll
-            for (int k = 0; k < kVT / 2; ++k) {
-                const ulonglong2 q = __ldg(p + k);
-                o[2 * k] = (OffT)q.x; o[2 * k + 1] = (OffT)q.y;
-            }
-        }
-        o[kVT] = __ldg(off + v0 + kVT);
-    } else {
-#pragma unroll
-        for (int k = 0; k <= kVT; ++k) o[k] = (v0 + k <= n) ? __ldg(off + v0 + k) : (OffT)0;
-    }
-}
+constexpr int kWPW = 64;                                  // bitmap words per warp per tile
+constexpr int kG = 8;                                     // words whose loads are in flight together
+constexpr uint32_t kScanV = (uint32_t)kWarps * kWPW * 32; // vertices per scan tile (16384)
 
 template <class OffT, bool UDC, bool BFSLAB>
 __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraphConditionalHandle cond,
@@ -338,12 +314,13 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
     __shared__ u64 s_wsum[kWarps];
     Ctl *ctl = d.ctl;
     const uint32_t epoch = ctl->epoch & 0x3FFFFFFFu;
-    const uint32_t n = d.n;
-    const uint32_t nscan = (n + kScanV - 1) / kScanV;
+    const uint32_t nscan = (d.n + kScanV - 1) / kScanV;
     const uint32_t ts = d.ts, tsl = d.ts_log2;
-    const uint32_t lane = lane_id();
+    const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
+    const uint32_t lt = (1u << lane) - 1u;
     uint32_t *label = ctl->label;
-    const uint32_t new_depth = ctl->depth + 1;      // BFS depth of the vertices in Q
+    const uint32_t new_depth = ctl->depth + 1;            // BFS depth of the vertices in Q
+    const uint32_t th = ctl->thresh;                      // near-far threshold (SSSP option)
     for (;;) {
         if (threadIdx.x == 0) s_tile = atomicAdd(&ctl->scan_ctr, 1u);
         __syncwarp();
@@ -351,49 +328,94 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
         const uint32_t tile = s_tile;
         __syncthreads();                                  // all have read s_tile before it is reused
         if (tile >= nscan) break;
-        const uint32_t v0 = tile * kScanV + threadIdx.x * kVT;
-        // this thread's bitmap word (read and cleared)
-        uint32_t bits = v0 < n ? d.Q[v0 >> 5] : 0u;
-        uint32_t far_bits = 0, far_min = kInf;
-        if (bits && d.nf_delta) {
-            // near-far SSSP: marked vertices at distance >= thresh stay marked
-            // (deferred, still active) and are not expanded in this iteration
-            const uint32_t th = ctl->thresh;
-            for (uint32_t b = bits; b; b &= b - 1) {
-                const uint32_t k = __ffs(b) - 1;
-                const uint32_t lv = __ldcg(&label[v0 + k]);
-                d.snap[v0 + k] = lv;                          // refresh the pre-filter snapshot
-                if (lv >= th) {
-                    far_bits |= 1u << k;
-                    far_min = min(far_min, lv);
-                }
-            }
-            bits &= ~far_bits;
-        }
-        if (bits | far_bits) d.Q[v0 >> 5] = far_bits;
-        if (d.nf_delta) {
-            const uint32_t fc = __reduce_add_sync(kFull, (uint32_t)__popc(far_bits));
-            const uint32_t fm = __reduce_min_sync(kFull, far_min);
-            if (lane == 0 && fc) {
-                atomicAdd(&ctl->far_count, fc);
-                atomicMin(&ctl->far_min, fm);
-            }
-            __threadfence();                                  // before this tile publishes
-        }
-        OffT o[kVT + 1];
-        u64 tsum = 0;
-        if (bits) {
-            load_offsets<OffT>(d.off, v0, n, o);
+        const uint32_t wbase = (tile * kWarps + warp) * kWPW;          // first word of this warp
+        // this warp's words: lane l holds words wbase + l + 32j (read, then cleared
+        // -- near-far SSSP keeps the deferred far bits)
+        uint32_t wq[kWPW / 32];
 #pragma unroll
-            for (int k = 0; k < kVT; ++k) {
-                if (bits & (1u << k)) {
-                    const uint32_t c = udc_count<UDC>((OffT)(o[k + 1] - o[k]), d.K);
-                    tsum += ((u64)(c > 0) << 32) | c;
+        for (int j = 0; j < kWPW / 32; ++j) wq[j] = d.Q[wbase + 32 * j + lane];
+        uint32_t far_cnt = 0, far_min = kInf;
+        if (d.nf_delta) {
+            // near-far: marked vertices with label >= thresh stay marked (deferred)
+#pragma unroll
+            for (int j = 0; j < kWPW / 32; ++j) {
+                uint32_t keep_far = 0;
+                for (uint32_t k = 0; k < 32; ++k) {
+                    const uint32_t word = __shfl_sync(kFull, wq[j], k);
+                    if (!word) continue;
+                    const bool bit = (word >> lane) & 1u;
+                    const uint32_t v = (wbase + 32 * j + k) * 32 + lane;
+                    uint32_t lv = 0;
+                    if (bit) {
+                        lv = __ldcg(&label[v]);
+                        d.snap[v] = lv;                   // refresh the pre-filter snapshot
+                    }
+                    const uint32_t far = __ballot_sync(kFull, bit && lv >= th);
+                    if (far) {
+                        if (bit && lv >= th) far_min = min(far_min, lv);
+                        if (lane == k) keep_far = far;
+                    }
+                    far_cnt += __popc(far);
+                }
+                if (wq[j] | keep_far) d.Q[wbase + 32 * j + lane] = keep_far;
+                wq[j] &= ~keep_far;
+            }
+            far_min = __reduce_min_sync(kFull, far_min);
+            if (lane == 0 && far_cnt) {
+                atomicAdd(&ctl->far_count, far_cnt);
+                atomicMin(&ctl->far_min, far_min);
+            }
+            __threadfence();                              // before this tile publishes
+        } else {
+#pragma unroll
+            for (int j = 0; j < kWPW / 32; ++j)
+                if (wq[j]) d.Q[wbase + 32 * j + lane] = 0u;
+        }
+        // pass 1: this warp's (kept, shadows); groups of kG words, all offset
+        // loads of a group issued before use
+        u64 wsum = 0;
+        uint32_t nbits = 0;
+#pragma unroll
+        for (int j = 0; j < kWPW / 32; ++j) {
+            for (uint32_t k0 = 0; k0 < 32; k0 += kG) {
+                uint32_t word[kG], any = 0;
+#pragma unroll
+                for (int r = 0; r < kG; ++r) {
+                    word[r] = __shfl_sync(kFull, wq[j], k0 + r);
+                    any |= word[r];
+                }
+                if (!any) continue;
+                OffT ob[kG], oe[kG];
+#pragma unroll
+                for (int r = 0; r < kG; ++r) {
+                    ob[r] = 0;
+                    oe[r] = 0;
+                    if ((word[r] >> lane) & 1u) {
+                        const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
+                        ob[r] = __ldg(&d.off[v]);
+                        oe[r] = __ldg(&d.off[v + 1]);
+                    }
+                }
+#pragma unroll
+                for (int r = 0; r < kG; ++r) {
+                    if (!word[r]) continue;
+                    nbits += __popc(word[r]);
+                    const uint32_t c = ((word[r] >> lane) & 1u) ? udc_count<UDC>((uint32_t)(oe[r] - ob[r]), d.K) : 0u;
+                    const uint32_t kept = __ballot_sync(kFull, c > 0);
+                    wsum += ((u64)__popc(kept) << 32) | __reduce_add_sync(kFull, c);
                 }
             }
         }
-        u64 btotal;
-        const u64 tprefix = block_excl_scan<u64>(tsum, s_wsum, btotal);
+        // block scan over the warps (warp order = vertex order)
+        if (lane == 0) s_wsum[warp] = wsum;
+        __syncwarp();
+        __syncthreads();
+        u64 wprefix = 0, btotal = 0;
+        for (int k = 0; k < kWarps; ++k) {
+            const u64 x = s_wsum[k];
+            if (k < (int)warp) wprefix += x;
+            btotal += x;
+        }
         if (threadIdx.x < 32) {
             u64 excl = 0;
             if (tile == 0) {
@@ -437,33 +459,59 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
             __syncwarp();
         }
         __syncthreads();
-        // pass 2: write the compacted entries (offsets still in registers)
-        if (bits) {
-            u64 run = s_prefix + tprefix;
+        // pass 2: write the compacted entries, in vertex order, coalesced
+        u64 run = s_prefix + wprefix;
 #pragma unroll
-            for (int k = 0; k < kVT; ++k) {
-                if (bits & (1u << k)) {
-                    const uint32_t v = v0 + k;
-                    if (BFSLAB) label[v] = new_depth;      // BFS: depth written once, on compaction
-                    else if (label && !d.nf_delta) d.snap[v] = __ldcg(&label[v]);   // refresh the snapshot
-                    const uint32_t dg = (uint32_t)(o[k + 1] - o[k]);
-                    const uint32_t c = udc_count<UDC>(dg, d.K);
+        for (int j = 0; j < kWPW / 32; ++j) {
+            for (uint32_t k0 = 0; k0 < 32; k0 += kG) {
+                uint32_t word[kG], any = 0;
+#pragma unroll
+                for (int r = 0; r < kG; ++r) {
+                    word[r] = __shfl_sync(kFull, wq[j], k0 + r);
+                    any |= word[r];
+                }
+                if (!any) continue;
+                OffT ob[kG], oe[kG];
+                uint32_t lv[kG];
+#pragma unroll
+                for (int r = 0; r < kG; ++r) {
+                    ob[r] = 0;
+                    oe[r] = 0;
+                    lv[r] = 0;
+                    if ((word[r] >> lane) & 1u) {
+                        const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
+                        ob[r] = __ldg(&d.off[v]);
+                        oe[r] = __ldg(&d.off[v + 1]);
+                        if (!BFSLAB && label && !d.nf_delta) lv[r] = __ldcg(&label[v]);
+                    }
+                }
+#pragma unroll
+                for (int r = 0; r < kG; ++r) {
+                    if (!word[r]) continue;
+                    const bool bit = (word[r] >> lane) & 1u;
+                    const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
+                    if (bit) {
+                        if (BFSLAB) label[v] = new_depth;         // BFS: depth written once, on compaction
+                        else if (label && !d.nf_delta) d.snap[v] = lv[r];   // refresh the snapshot
+                    }
+                    const uint32_t dg = (uint32_t)(oe[r] - ob[r]);
+                    const uint32_t c = bit ? udc_count<UDC>(dg, d.K) : 0u;
+                    const uint32_t kept = __ballot_sync(kFull, c > 0);
+                    const uint32_t cincl = warp_incl_scan(c);
                     if (c) {
-                        const uint32_t pos = (uint32_t)(run >> 32);
-                        const uint32_t sh = (uint32_t)run;
+                        const uint32_t pos = (uint32_t)(run >> 32) + __popc(kept & lt);
+                        const uint32_t sh = (uint32_t)run + cincl - c;
                         d.F[pos] = v;
-                        d.B[pos] = o[k];
+                        d.B[pos] = ob[r];
                         d.D[pos] = dg;
                         d.S[pos] = sh;
                         // tiles whose first shadow t*ts lies in [sh, sh + c)
                         for (uint32_t t = (sh + ts - 1) >> tsl; (t << tsl) < sh + c; ++t) d.tile_first[t] = pos;
-                        run += ((u64)1 << 32) | c;
                     }
+                    run += ((u64)__popc(kept) << 32) | __shfl_sync(kFull, cincl, 31);
                 }
             }
         }
-        // activations: one atomic per warp
-        const uint32_t nbits = __reduce_add_sync(kFull, (uint32_t)__popc(bits));
         if (lane == 0 && nbits) atomicAdd(&ctl->activations, (u64)nbits);   // result unused: RED
         if (tile == nscan - 1 && threadIdx.x == 0) {
             const u64 total = s_prefix + btotal;
@@ -478,8 +526,8 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
             if (d.nf_delta && ctl->far_count) {
                 more = true;
                 if (nF == 0) {                        // near set empty: next bucket
-                    const unsigned long long th = (unsigned long long)ctl->far_min + d.nf_delta;
-                    ctl->thresh = th > kInf ? kInf : (uint32_t)th;
+                    const unsigned long long thn = (unsigned long long)ctl->far_min + d.nf_delta;
+                    ctl->thresh = thn > kInf ? kInf : (uint32_t)thn;
                 }
             }
             ctl->more = more ? 1u : 0u;
