@@ -60,6 +60,8 @@ def parse_args():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-profile", action="store_true")
     p.add_argument("--json-out", default=None)
+    p.add_argument("--host-edges", action="store_true",
+                   help="NEXT-2: keep col/w in pinned host memory (zero-copy reads by the kernels)")
     p.add_argument("--partitioned", action="store_true",
                    help="1-D destination partition of ONE graph over the N ranks (NCCL exchange); "
                         "default: N independent replicas")
@@ -324,6 +326,10 @@ def run_ours(args):
 
     def mk(graph, flags, sym=False):
         o, c, w, fl = etg.csr_to_device(graph.off, graph.col, graph.w, device=dev)
+        if args.host_edges:
+            c = c.cpu().pin_memory()
+            w = None if w is None else w.cpu().pin_memory()
+            fl |= etg.HOST_EDGES
         return etg.Graph(o, c, w, n=graph.n, K=args.K, flags=flags | fl | args.flags, symmetric=sym,
                          sssp_delta=args.sssp_delta)
 

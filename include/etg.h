@@ -69,8 +69,12 @@ enum {
                                   iteration) instead of a CUDA-graph conditional while node */
     ETG_PROFILE = 1u << 6,     /* implies ETG_HOST_LOOP; CUDA events around every scan and
                                   expand launch on the handle's stream fill scan_ms/expand_ms */
-    ETG_SMP_SHARED = 1u << 7   /* SMP as literally described (L199): TMA bulk copies of the next
+    ETG_SMP_SHARED = 1u << 7,  /* SMP as literally described (L199): TMA bulk copies of the next
                                   tile's segments into per-warp shared-memory stages (K <= 32) */
+    ETG_HOST_EDGES = 1u << 8   /* host-resident edge mode (NEXT-2; Sec. IV-B): d_col_idx
+                                  and d_weights point to pinned, device-mapped HOST memory (UVA
+                                  zero-copy); each iteration reads only the active vertices' edges
+                                  over the host link.  Offsets and workspace stay in HBM. */
 };
 
 typedef struct {

@@ -24,10 +24,12 @@ __all__ = [
     "EtgError", "Stats", "Graph", "load_csr", "csr_to_device", "to_u32_numpy",
     "run_host", "host_scratch_bytes", "kernel_launches", "lib",
     "SYMMETRIC", "NO_UDC", "NO_SMP", "OFFSETS_U64", "VALIDATE", "HOST_LOOP", "PROFILE", "SMP_SHARED",
+    "HOST_EDGES",
     "INF", "CAP", "BFS", "SSSP", "CC", "SSWP",
 ]
 
-SYMMETRIC, NO_UDC, NO_SMP, OFFSETS_U64, VALIDATE, HOST_LOOP, PROFILE, SMP_SHARED = 1, 2, 4, 8, 16, 32, 64, 128
+SYMMETRIC, NO_UDC, NO_SMP, OFFSETS_U64, VALIDATE, HOST_LOOP, PROFILE, SMP_SHARED, HOST_EDGES = (
+    1, 2, 4, 8, 16, 32, 64, 128, 256)
 INF, CAP = 0xFFFFFFFF, 0xFFFFFFFE
 BFS, SSSP, CC, SSWP = 0, 1, 2, 3
 
@@ -165,8 +167,13 @@ class Graph:
         if col.dtype != torch.int32 or (w is not None and w.dtype != torch.int32):
             raise EtgError("col and w must be int32 tensors holding uint32 bits")
         for t in (off, col, w):
-            if t is not None and (not t.is_cuda or not t.is_contiguous()):
-                raise EtgError("CSR tensors must be contiguous CUDA tensors")
+            if t is None:
+                continue
+            edge_array = t is not off
+            host_ok = edge_array and (flags & HOST_EDGES) and t.is_pinned()
+            if not t.is_contiguous() or not (t.is_cuda or host_ok):
+                raise EtgError("CSR tensors must be contiguous CUDA tensors "
+                               "(col/w may be pinned host tensors with HOST_EDGES)")
         if symmetric:
             flags |= SYMMETRIC
         if validate:
@@ -176,6 +183,8 @@ class Graph:
         self.K = K
         self.flags = flags
         self.device = off.device
+        if not off.is_cuda:
+            raise EtgError("row offsets must live on the device")
         self._keep = (off, col, w)
         self._stream = stream
         self._opt = Options(K, flags, sssp_delta)

@@ -84,8 +84,9 @@ Params derive(const etg_options *opt, uint32_t tune) {
         // 32 * (K + 6) words, affordable in shared memory for K <= 32
         p.ts = 32;
         p.idx = false;
-        p.smp = p.udc && (flags & ETG_SMP_SHARED) && !(flags & ETG_NO_SMP) && p.K <= 32;
-        p.prefetch = p.udc && !(flags & ETG_NO_SMP) && !p.smp;
+        const bool host_edges = (flags & ETG_HOST_EDGES) != 0;   // no TMA on host-mapped memory
+        p.smp = p.udc && (flags & ETG_SMP_SHARED) && !(flags & ETG_NO_SMP) && p.K <= 32 && !host_edges;
+        p.prefetch = p.udc && !(flags & ETG_NO_SMP) && !p.smp && !host_edges;
     }
     p.ts_log2 = 0;
     while ((1u << p.ts_log2) < p.ts) ++p.ts_log2;

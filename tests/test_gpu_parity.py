@@ -288,3 +288,28 @@ def test_sssp_near_far_schedule(c1, delta):
     off, col, w = g.numpy()
     s = gg.first_source(g)
     np.testing.assert_array_equal(U32(to_etg(g, sssp_delta=delta).sssp(s)[0]), oracle.sssp(off, col, w, s))
+
+
+def test_host_resident_edges(c1):
+    """NEXT-2: col/w in pinned host memory, read zero-copy by the kernels."""
+    off, col, w = c1.numpy()
+    o, c, ww, fl = etg.csr_to_device(c1.off, c1.col, c1.w, device="cuda")
+    ch, wh = c.cpu().pin_memory(), ww.cpu().pin_memory()
+    G = etg.Graph(o, ch, wh, n=c1.n, flags=fl | etg.HOST_EDGES)
+    for s in gg.sample_sources(c1, 2, 77):
+        np.testing.assert_array_equal(U32(G.bfs(s)[0]), oracle.bfs(off, col, s))
+        np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
+
+
+def test_galois_gr_file_traversal(tmp_path, c1):
+    """NEXT-4: a .gr file written from C1, read back, traversed on the GPU."""
+    from paper_conf_ipps_wangzlg19_b200 import gr
+    off, col, w = c1.numpy()
+    p = str(tmp_path / "c1.gr")
+    gr.write_gr(p, off.astype(np.int64), col, w)
+    o2, c2, w2 = gr.read_gr(p)
+    od, cd, wd, fl = etg.csr_to_device(torch.from_numpy(o2), torch.from_numpy(c2.astype(np.int64)),
+                                       torch.from_numpy(w2.astype(np.int64)), device="cuda")
+    G = etg.Graph(od, cd, wd, n=c1.n, flags=fl, validate=True)
+    s = gg.first_source(c1)
+    np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))

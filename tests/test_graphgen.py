@@ -90,3 +90,28 @@ def test_bucketed_dedup_is_equivalent(monkeypatch):
     monkeypatch.setattr(gg, "_BUCKET_TUPLES", 1 << 27)
     d = gg.make("LJ-small", weights=False)
     assert c.sha256() == d.sha256()
+
+
+def test_galois_gr_roundtrip(tmp_path):
+    """NEXT-4: the .gr reader/writer round-trips CSR + weights, v1 and v2."""
+    from paper_conf_ipps_wangzlg19_b200 import gr
+    g = gg.make("T12")
+    off, col, w = g.numpy()
+    for version in (1, 2):
+        for weights in (None, w):
+            p = str(tmp_path / f"g{version}{weights is None}.gr")
+            gr.write_gr(p, off.astype(np.int64), col, weights, version=version)
+            o2, c2, w2 = gr.read_gr(p)
+            assert np.array_equal(o2, off.astype(np.int64)) and np.array_equal(c2, col)
+            assert (w2 is None) == (weights is None)
+            if weights is not None:
+                assert np.array_equal(w2, w)
+    odd = gg.from_edges("odd", 3, [(0, 1), (1, 2), (2, 0)])
+    o, c, _ = odd.numpy()
+    p = str(tmp_path / "odd.gr")
+    gr.write_gr(p, o.astype(np.int64), c)                 # m odd: v1 pads to 8 bytes
+    assert np.array_equal(gr.read_gr(p)[1], c)
+    with open(p, "r+b") as f:                               # corrupt the size
+        f.truncate(40)
+    with pytest.raises(ValueError):
+        gr.read_gr(p)
