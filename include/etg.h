@@ -178,6 +178,12 @@ etg_status etg_step_expand(etg_graph *g);
 etg_status etg_step_scan(etg_graph *g, uint32_t *n_active);
 etg_status etg_step_end(etg_graph *g, etg_stats *st_or_null);
 etg_status etg_bitmap_layout(etg_graph *g, size_t *offset_bytes, uint32_t *nwords);
+/* Tracing (step-wise runs): the device counters as of the last etg_step_* call
+ * that synchronised (begin/scan/end): out[0] depth, [1] compacted active-set
+ * size |F| (Proc. 1 actSet, L207), [2] shadow vertices of F (Def. 3),
+ * [3] cumulative edges expanded, [4] cumulative activations, [5] iterations.
+ * `out` is host memory of 6 entries.  ETG_EINVAL on NULL arguments. */
+etg_status etg_debug_counters(etg_graph *g, uint64_t *out);
 
 /* Release a handle (does not free the borrowed device memory). */
 void etg_free(etg_graph *g);

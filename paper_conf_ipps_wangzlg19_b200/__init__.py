@@ -87,6 +87,7 @@ def lib():
             "etg_kernel_launches": (u64, []),
             "etg_step_begin": (st, [p, ctypes.c_int, u32, p, ctypes.POINTER(u32)]),
             "etg_step_expand": (st, [p]),
+            "etg_debug_counters": (st, [p, ctypes.POINTER(ctypes.c_uint64)]),
             "etg_step_scan": (st, [p, ctypes.POINTER(u32)]),
             "etg_step_end": (st, [p, p]),
             "etg_bitmap_layout": (st, [p, ctypes.POINTER(sz), ctypes.POINTER(u32)]),

@@ -816,4 +816,16 @@ const char *etg_last_error(void) { return g_err.c_str(); }
 
 uint64_t etg_kernel_launches(void) { return g_launches.load(); }
 
+etg_status etg_debug_counters(etg_graph *g, uint64_t *out) {
+    if (!g || !out) return fail(ETG_EINVAL, "null handle or output");
+    const Ctl &c = *g->h_ctl;
+    out[0] = c.depth;
+    out[1] = c.nF;
+    out[2] = c.nshadow;
+    out[3] = c.edges;
+    out[4] = c.activations;
+    out[5] = c.iterations;
+    return ETG_OK;
+}
+
 }  // extern "C"
