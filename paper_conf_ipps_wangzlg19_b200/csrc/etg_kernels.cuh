@@ -108,6 +108,7 @@ constexpr uint32_t kTuneFilterL1 = 1u;    // pre-filter label loads cached in L1
 // replay-only experiment switches (etg_debug_expand_replay; results not kept)
 constexpr uint32_t kTuneNoGather = 16u;   // skip the label gather and the commit
 constexpr uint32_t kTuneNoCommit = 32u;   // gather labels but never commit (counts passes)
+constexpr uint32_t kTuneQMark = 64u;      // A/B: SSSP/CC/SSWP commits also set Q, the scan reads only Q
 
 // ------------------------------------------------------------------------- //
 // small device helpers
@@ -301,9 +302,13 @@ __global__ __launch_bounds__(kBlock) void init_kernel(Dev<OffT> d, uint32_t *lab
 // (kept entries << 32 | shadows); neither half can carry into the other
 // (entries <= n < 2^32, shadows < 2^32 checked at load time).
 // ------------------------------------------------------------------------- //
-constexpr int kWPW = 64;                                  // bitmap words per warp per tile
+#ifndef ETG_WPW
+#define ETG_WPW 32
+#endif
+constexpr int kWPW = ETG_WPW;                             // bitmap words per warp per tile
 constexpr int kG = 8;                                     // words whose loads are in flight together
-constexpr uint32_t kScanV = (uint32_t)kWarps * kWPW * 32; // vertices per scan tile (16384)
+constexpr uint32_t kScanV = (uint32_t)kWarps * kWPW * 32; // vertices per scan tile (8192)
+constexpr int kLB = 4;                                    // look-back window: 32 * kLB predecessor tiles
 
 template <class OffT, bool UDC, bool BFSLAB>
 __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraphConditionalHandle cond,
@@ -321,6 +326,7 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
     uint32_t *label = ctl->label;
     const uint32_t new_depth = ctl->depth + 1;            // BFS depth of the vertices in Q
     const uint32_t th = ctl->thresh;                      // near-far threshold (SSSP option)
+    const bool qmark = !d.nf_delta && (d.tune & kTuneQMark);   // A/B switch: the expand marks Q itself
     for (;;) {
         if (threadIdx.x == 0) s_tile = atomicAdd(&ctl->scan_ctr, 1u);
         __syncwarp();
@@ -370,6 +376,36 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
 #pragma unroll
             for (int j = 0; j < kWPW / 32; ++j)
                 if (wq[j]) d.Q[wbase + 32 * j + lane] = 0u;
+            if (!BFSLAB && label && !(d.tune & kTuneQMark)) {
+                // SSSP/CC/SSWP: a vertex is active iff its label moved since it
+                // was last expanded (label != snap; the expand marks nothing for
+                // them), or init/exchange put it in Q.  Word k of the warp = the
+                // ballot over vertices 32k .. 32k+31: coalesced label/snap loads.
+#pragma unroll
+                for (int j = 0; j < kWPW / 32; ++j) {
+                    uint32_t mine = 0;
+                    for (uint32_t k0 = 0; k0 < 32; k0 += 2 * kG) {
+                        uint32_t lv[2 * kG], sv[2 * kG];
+#pragma unroll
+                        for (int r = 0; r < 2 * kG; ++r) {
+                            const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
+                            lv[r] = 0;
+                            sv[r] = 0;
+                            if (v < d.n) {
+                                lv[r] = __ldcg(&label[v]);
+                                sv[r] = __ldcg(&d.snap[v]);
+                            }
+                        }
+#pragma unroll
+                        for (int r = 0; r < 2 * kG; ++r) {
+                            const uint32_t b = __ballot_sync(kFull, lv[r] != sv[r]);
+                            if (lane == k0 + r) mine = b;
+                            if (lv[r] != sv[r]) d.snap[(wbase + 32 * j + k0 + r) * 32 + lane] = lv[r];   // refresh
+                        }
+                    }
+                    wq[j] |= mine;
+                }
+            }
         }
         // pass 1: this warp's (kept, shadows); groups of kG words, all offset
         // loads of a group issued before use
@@ -430,24 +466,53 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
                     __threadfence();
                     atomicExch(&d.st_flag[tile], (epoch << 2) | 1u);
                 }
-                int p = (int)tile - 1;                  // nearest predecessor in lane 0
+                // Window of 32 * kLB predecessors, all flag loads in flight at
+                // once: position i = 32k + lane is tile p - i.  Aggregates are
+                // published before any look-back, so a tile sums them directly
+                // up to the nearest inclusive prefix without waiting for its
+                // neighbours' look-backs (one round trip for <= 32 * kLB tiles).
+                int p = (int)tile - 1;                  // nearest predecessor at position 0
                 for (;;) {
-                    const int q = p - (int)lane;
-                    uint32_t f = (epoch << 2) | 1u;     // q < 0: beyond tile 0, never needed
-                    if (q >= 0) f = ld_volatile_u32(&d.st_flag[q]);
-                    const bool valid = (f >> 2) == epoch && (f & 3u) != 0;
-                    const uint32_t incl = __ballot_sync(kFull, valid && (f & 3u) == 2u && q >= 0);
-                    const uint32_t inval = __ballot_sync(kFull, !valid);
-                    const uint32_t first = incl ? (uint32_t)(__ffs(incl) - 1) : 32u;
-                    const uint32_t need = first < 31 ? ((2u << first) - 1u) : kFull;
-                    if (inval & need) continue;         // a needed predecessor is not published yet
+                    uint32_t f[kLB];
+#pragma unroll
+                    for (int k = 0; k < kLB; ++k) {
+                        const int q = p - (int)lane - 32 * k;
+                        f[k] = (epoch << 2) | 1u;       // q < 0: beyond tile 0, contributes 0
+                        if (q >= 0) f[k] = ld_volatile_u32(&d.st_flag[q]);
+                    }
+                    int firstk = kLB;                   // window row of the nearest inclusive prefix
+                    uint32_t first = 32;                //   and its lane
+                    bool wait = false;
+#pragma unroll
+                    for (int k = 0; k < kLB; ++k) {
+                        const int q = p - (int)lane - 32 * k;
+                        const bool valid = (f[k] >> 2) == epoch && (f[k] & 3u) != 0;
+                        const uint32_t incl = __ballot_sync(kFull, valid && (f[k] & 3u) == 2u && q >= 0);
+                        const uint32_t inval = __ballot_sync(kFull, !valid);
+                        if (firstk == kLB) {
+                            if (incl) {
+                                firstk = k;
+                                first = (uint32_t)(__ffs(incl) - 1);
+                                const uint32_t need = first < 31 ? ((2u << first) - 1u) : kFull;
+                                if (inval & need) wait = true;
+                            } else if (inval) {
+                                wait = true;
+                            }
+                        }
+                    }
+                    if (wait) continue;                 // a needed predecessor is not published yet
                     __threadfence();
                     u64 val = 0;
-                    if (lane < first && q >= 0) val = ld_volatile_u64(&d.st_agg[q]);
-                    else if (lane == first) val = ld_volatile_u64(&d.st_inc[q]);
+#pragma unroll
+                    for (int k = 0; k < kLB; ++k) {
+                        const int q = p - (int)lane - 32 * k;
+                        if (q < 0) continue;
+                        if (k < firstk || (k == firstk && lane < first)) val += ld_volatile_u64(&d.st_agg[q]);
+                        else if (k == firstk && lane == first) val += ld_volatile_u64(&d.st_inc[q]);
+                    }
                     excl += warp_sum_u64(val);
-                    if (first < 32) break;
-                    p -= 32;
+                    if (firstk < kLB) break;
+                    p -= 32 * kLB;
                 }
                 if (lane == 0) {
                     d.st_inc[tile] = excl + btotal;
@@ -482,7 +547,7 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
                         const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
                         ob[r] = __ldg(&d.off[v]);
                         oe[r] = __ldg(&d.off[v + 1]);
-                        if (!BFSLAB && label && !d.nf_delta) lv[r] = __ldcg(&label[v]);
+                        if (!BFSLAB && label && qmark) lv[r] = __ldcg(&label[v]);
                     }
                 }
 #pragma unroll
@@ -492,7 +557,7 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
                     const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
                     if (bit) {
                         if (BFSLAB) label[v] = new_depth;         // BFS: depth written once, on compaction
-                        else if (label && !d.nf_delta) d.snap[v] = lv[r];   // refresh the snapshot
+                        else if (label && qmark) d.snap[v] = lv[r];   // refresh the snapshot (Q-mark mode)
                     }
                     const uint32_t dg = (uint32_t)(oe[r] - ob[r]);
                     const uint32_t c = bit ? udc_count<UDC>(dg, d.K) : 0u;
@@ -615,12 +680,15 @@ __device__ __forceinline__ bool improves(uint32_t cand, uint32_t cur) {
 // thread's value wins (reading R-5: the bitmap de-duplicates).  BFS only sets
 // the bit: every discoverer of u in this iteration would write the same depth,
 // and the scan that compacts u writes it once.
+// SSSP/CC/SSWP set no bit: the scan finds the moved labels by comparing them
+// with the iteration-start snapshot (one random access per commit instead of
+// two); only the near-far schedule, which defers marks in Q, still sets it.
 template <int ALG>
 __device__ __forceinline__ void commit(uint32_t *label, uint32_t *Q, uint32_t u, uint32_t cand,
-                                       uint64_t pol) {
+                                       uint64_t pol, bool markQ) {
     if (ALG == ALG_SSWP) red_max(&label[u], cand, pol);
     else if (ALG != ALG_BFS) red_min(&label[u], cand, pol);
-    red_or(&Q[u >> 5], 1u << (u & 31), pol);
+    if (ALG == ALG_BFS || markQ) red_or(&Q[u >> 5], 1u << (u & 31), pol);
 }
 
 // ------------------------------------------------------------------------- //
@@ -743,7 +811,7 @@ __global__ __launch_bounds__(kBlock) void expand_kernel(Dev<OffT> d, uint32_t ca
                 cur[r] = act[r] ? (l1 ? ld_ca(&label[u[r]]) : ld_cg(&label[u[r]])) : 0u;
 #pragma unroll
             for (int r = 0; r < kR; ++r)
-                if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep);
+                if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, d.nf_delta != 0 || (d.tune & kTuneQMark));
         }
         my_edges += E;
         __syncthreads();
@@ -1041,7 +1109,7 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
                 }
 #pragma unroll
                 for (int r = 0; r < kR; ++r)
-                    if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep);
+                    if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, d.nf_delta != 0 || (d.tune & kTuneQMark));
             }
             if (tn >= ntiles) break;
         }

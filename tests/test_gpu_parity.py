@@ -130,6 +130,18 @@ def test_flag_invariance(c1, c1sym, flags):
     check_cc(c1sym, flags=flags)
 
 
+@pytest.mark.parametrize("tune", [64, 2, 2 | 64])
+def test_engine_variants(c1, c1sym, monkeypatch, tune):
+    """Engine variants picked at load time (ETG_TUNE): 64 = SSSP/CC/SSWP commits mark the
+    bitmap and the scan reads only it (no label/snapshot comparison);
+    2 = the CTA-tile expand kernel.  Labels are the same unique fixpoints."""
+    monkeypatch.setenv("ETG_TUNE", str(tune))
+    srcs = gg.sample_sources(c1, 2, 17)
+    check_all(c1, srcs)
+    check_cc(c1sym)
+    check_cc(c1sym, flags=32)
+
+
 def test_u64_offsets(c1):
     check_all(c1, gg.sample_sources(c1, 2, 3), force_u64=True)
 
