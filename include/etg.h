@@ -85,7 +85,8 @@ typedef struct {
                                 improved vertices at distance >= a threshold stay active but are
                                 deferred; the threshold advances by sssp_delta when no nearer
                                 vertex is active.  Same distances (unique fixpoint), fewer
-                                redundant relaxations.  Ignored by the step-wise (multi-GPU) API. */
+                                redundant relaxations.  The step-wise (multi-GPU) API honours it
+                                too: the deferred vertices stay in the exchanged bitmap. */
 } etg_options;
 
 typedef struct {

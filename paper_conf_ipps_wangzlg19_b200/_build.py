@@ -8,7 +8,7 @@ import subprocess
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
-LIB = os.path.join(HERE, "libetg.so")
+LIB = os.environ.get("ETG_LIB_PATH") or os.path.join(HERE, "libetg.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 NVCC_FLAGS = [
@@ -39,7 +39,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, *NVCC_FLAGS, *sources(), "-o", tmp]
+    extra = os.environ.get("ETG_NVCC_EXTRA", "").split()   # experiment builds (e.g. -DETG_PIPE=0)
+    cmd = [NVCC, *NVCC_FLAGS, *extra, *sources(), "-o", tmp]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd))

@@ -94,7 +94,7 @@ Params derive(const etg_options *opt, uint32_t tune) {
 }
 
 struct Layout {
-    size_t Q, snap, F, B, D, S, tile_first, st_flag, st_agg, st_inc, ctl, total;
+    size_t Q, V, snap, F, B, D, S, tile_first, st_flag, st_agg, st_inc, ctl, total;
     uint32_t nwords;
 };
 
@@ -113,6 +113,7 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
     const uint64_t tile_words = kScanV / 32;
     L.nwords = (uint32_t)((words + tile_words - 1) / tile_words * tile_words);
     L.Q = take(4ull * L.nwords);
+    L.V = take(4ull * L.nwords);
     L.snap = take(4 * (n + 1));
     L.F = take(4 * (n + 1));
     L.B = take((p.u64 ? 8 : 4) * (n + 1));
@@ -164,6 +165,7 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.col = g->col;
     d.w = g->w;
     d.Q = reinterpret_cast<uint32_t *>(g->ws + g->L.Q);
+    d.V = reinterpret_cast<uint32_t *>(g->ws + g->L.V);
     d.nwords = g->L.nwords;
     d.snap = reinterpret_cast<uint32_t *>(g->ws + g->L.snap);
     d.F = reinterpret_cast<uint32_t *>(g->ws + g->L.F);
@@ -259,7 +261,10 @@ etg_status expand_launch(etg_graph *g, int alg, Launch &out) {
     out.fn = expand_fn_alg<OffT>(alg, g->p.udc, g->p.idx, g->p.smp, g->p.warp);
     out.smem = expand_smem(g->p, alg);
     ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)out.smem));
-    ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+    // no dynamic shared memory: leave the unified L1/shared array to L1 (the
+    // BFS visited bitmap is read through it); SMP stages: maximum shared memory
+    ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                out.smem ? 100 : 0));
     int nb = 0;
     ETG_CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, out.fn, kBlock, out.smem));
     if (nb < 1) nb = 1;
@@ -406,9 +411,10 @@ etg_status step_scan_impl(etg_graph *g, uint32_t *n_active);
 template <class OffT>
 etg_status step_begin_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, uint32_t *n_active,
                            int skip_scan) {
-    Dev<OffT> d = make_dev<OffT>(g);
+    Dev<OffT> d = make_dev<OffT>(g, alg);
     cudaStream_t s = g->stream;
     ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, label, source);
+    if (d.nf_delta) ctl_nearfar_kernel<<<1, 1, 0, s>>>(g->ctl, d.nf_delta);
     void *iargs[] = {&d, &label, &source};
     ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), iargs, 0, s));
     g->step_launches = 2;
@@ -422,16 +428,26 @@ etg_status step_begin_impl(etg_graph *g, int alg, uint32_t source, uint32_t *lab
 
 template <class OffT>
 etg_status step_scan_impl(etg_graph *g, uint32_t *n_active) {
-    Dev<OffT> d = make_dev<OffT>(g);
+    Dev<OffT> d = make_dev<OffT>(g, g->step_alg);
     cudaStream_t s = g->stream;
     cudaGraphConditionalHandle none = 0;
     int zero = 0;
     void *scan_args[] = {&d, &none, &zero};
-    ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, g->step_alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
-    g->step_launches += 1;
-    ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
-    ETG_CU(cudaStreamSynchronize(s));
-    ETG_CU(cudaGetLastError());
+    for (int rescan = 0;; ++rescan) {
+        if (rescan) {
+            ctl_rescan_kernel<<<1, 1, 0, s>>>(g->ctl);
+            g->step_launches += 1;
+        }
+        ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, g->step_alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+        g->step_launches += 1;
+        ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+        ETG_CU(cudaStreamSynchronize(s));
+        ETG_CU(cudaGetLastError());
+        // near-far: an empty near set with deferred vertices advanced the
+        // threshold; scan again (nothing changed in between) until some
+        // vertices are activated or none remain
+        if (!d.nf_delta || g->h_ctl->activations != g->step_acts || !g->h_ctl->more) break;
+    }
     // vertices activated (bits consumed) by this scan: the same on every rank
     *n_active = (uint32_t)(g->h_ctl->activations - g->step_acts);
     g->step_acts = g->h_ctl->activations;
@@ -440,7 +456,7 @@ etg_status step_scan_impl(etg_graph *g, uint32_t *n_active) {
 
 template <class OffT>
 etg_status step_expand_impl(etg_graph *g) {
-    Dev<OffT> d = make_dev<OffT>(g);
+    Dev<OffT> d = make_dev<OffT>(g, g->step_alg);
     Launch ex;
     etg_status rc = expand_launch<OffT>(g, g->step_alg, ex);
     if (rc != ETG_OK) return rc;

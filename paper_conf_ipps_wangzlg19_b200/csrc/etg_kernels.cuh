@@ -48,6 +48,9 @@ constexpr uint32_t kFull = 0xFFFFFFFFu;
 #ifndef ETG_MINB
 #define ETG_MINB 1
 #endif
+#ifndef ETG_PIPE
+#define ETG_PIPE 1                          // software-pipelined batch loop in the warp expand
+#endif
 constexpr int kR = ETG_KR;                  // edges (chunks) in flight per thread in the relax loop
 
 enum Alg : int { ALG_BFS = 0, ALG_SSSP = 1, ALG_CC = 2, ALG_SSWP = 3 };
@@ -83,6 +86,7 @@ struct Dev {
     const uint32_t *col;
     const uint32_t *w;
     uint32_t *Q;                // next-active-set bitmap (nwords words, zero between uses)
+    uint32_t *V;                // BFS: visited bitmap as of the iteration start (label != INF)
     uint32_t *snap;             // labels at the start of the iteration (SSSP/CC/SSWP pre-filter)
     uint32_t *F;                // compacted active set (vertex ids, ascending)
     OffT *B;                    // off[F[k]]
@@ -265,6 +269,15 @@ __global__ void ctl_begin_kernel(Ctl *ctl, uint32_t *label, uint32_t source) {
 // near-far SSSP: the first threshold (the source has distance 0)
 __global__ void ctl_nearfar_kernel(Ctl *ctl, uint32_t delta) { ctl->thresh = delta; }
 
+// the scan bookkeeping an expand launch does (see expand kernels), for a scan
+// that directly follows another scan (step-wise near-far: empty near set)
+__global__ void ctl_rescan_kernel(Ctl *ctl) {
+    ctl->scan_ctr = 0;
+    ctl->epoch += 1;
+    ctl->far_min = kInf;
+    ctl->far_count = 0;
+}
+
 // BFS/SSSP: label = INF, label[s] = 0, Q = {s}.  SSWP: label = 0, label[s] =
 // INF, Q = {s}.  CC: label[v] = v, Q = all vertices (the scan drops degree-0
 // ones).  Q is all-zero on entry (every scan clears what it reads).
@@ -279,6 +292,10 @@ __global__ __launch_bounds__(kBlock) void init_kernel(Dev<OffT> d, uint32_t *lab
         else lab = (v == source) ? 0u : kInf;
         label[v] = lab;
         if (ALG != ALG_BFS) d.snap[v] = lab;
+    }
+    if (ALG == ALG_BFS) {
+        for (uint32_t k = blockIdx.x * kBlock + threadIdx.x; k < d.nwords; k += stride)
+            d.V[k] = (k == (source >> 5)) ? (1u << (source & 31)) : 0u;
     }
     if (ALG == ALG_CC) {
         for (uint32_t k = blockIdx.x * kBlock + threadIdx.x; k < d.nwords; k += stride) {
@@ -317,7 +334,9 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
     __shared__ uint32_t s_tile;
     __shared__ u64 s_prefix;
     __shared__ u64 s_wsum[kWarps];
+    __shared__ uint32_t s_acts;                           // activations of this CTA (one global atomic)
     Ctl *ctl = d.ctl;
+    if (threadIdx.x == 0) s_acts = 0;
     const uint32_t epoch = ctl->epoch & 0x3FFFFFFFu;
     const uint32_t nscan = (d.n + kScanV - 1) / kScanV;
     const uint32_t ts = d.ts, tsl = d.ts_log2;
@@ -375,7 +394,10 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
         } else {
 #pragma unroll
             for (int j = 0; j < kWPW / 32; ++j)
-                if (wq[j]) d.Q[wbase + 32 * j + lane] = 0u;
+                if (wq[j]) {
+                    d.Q[wbase + 32 * j + lane] = 0u;
+                    if (BFSLAB) d.V[wbase + 32 * j + lane] |= wq[j];   // visited from now on (depth written below)
+                }
             if (!BFSLAB && label && !(d.tune & kTuneQMark)) {
                 // SSSP/CC/SSWP: a vertex is active iff its label moved since it
                 // was last expanded (label != snap; the expand marks nothing for
@@ -577,7 +599,7 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
                 }
             }
         }
-        if (lane == 0 && nbits) atomicAdd(&ctl->activations, (u64)nbits);   // result unused: RED
+        if (lane == 0 && nbits) atomicAdd(&s_acts, nbits);
         if (tile == nscan - 1 && threadIdx.x == 0) {
             const u64 total = s_prefix + btotal;
             const uint32_t nF = (uint32_t)(total >> 32), N = (uint32_t)total;
@@ -601,6 +623,7 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
         __syncwarp();
         __syncthreads();
     }
+    if (threadIdx.x == 0 && s_acts) atomicAdd(&ctl->activations, (u64)s_acts);   // result unused: RED
 }
 
 // ------------------------------------------------------------------------- //
@@ -1025,6 +1048,144 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
         return w;
     };
 
+#if ETG_PIPE
+    // Software pipeline over the warp's stream of batches (kR chunks of 32
+    // elements; a tile is one or more batches).  Stage A of batch b+1 (owner
+    // masks, column/weight loads, candidates) is issued before stage B of batch
+    // b (label gathers, commits), so the column loads of the next batch are in
+    // flight while the gathers of this one are: one memory latency per batch
+    // instead of two.  Stage B needs only registers, so a tile's shared-memory
+    // stage (SMP) can be refilled once stage A has left the tile.
+    const bool markQ = d.nf_delta != 0 || (d.tune & kTuneQMark);
+    const uint32_t *filt = (ALG == ALG_BFS) ? label : d.snap;   // BFS: live labels; else snapshot (R-4, R-6)
+    uint32_t t = next_tile();
+    if (t < ntiles) {
+        WarpTile<OffT, UDC> nxt = prepare(t, 0);
+        // stage-A cursor: tile A_t (sequence number kt), batch start A_x0
+        WarpTile<OffT, UDC> A_t = nxt;
+        uint32_t kt = 0;
+        uint32_t tn = next_tile();
+        if (tn < ntiles) nxt = prepare(tn, 1);
+        uint32_t A_lab = (ALG == ALG_BFS) ? level : (A_t.sh.len ? ld_cg(&label[A_t.sh.v]) : 0u);
+        uint32_t A_x0 = 0, A_owner = 0xFFFFFFFFu;
+        const uint32_t *A_sbuf = nullptr;
+        if (SMP) {
+            mbar_wait(&bars[0], 0);
+            __syncwarp();
+            A_sbuf = wbuf;
+        }
+        my_edges += A_t.E;
+        bool A_valid = true;
+        uint32_t u0[kR], c0[kR], u1[kR], c1[kR];
+        uint32_t am0 = 0, am1 = 0;
+        // stage A: the batch at (A_t, A_x0) into (u, c, am); then advance the cursor
+        auto stage_a = [&](uint32_t (&u)[kR], uint32_t (&c)[kR], uint32_t &am) {
+            const uint32_t pos = A_t.o - A_x0;                 // this lane's slice start in the batch
+            const bool in_win = A_t.sh.len && pos < 32u * kR;
+            uint32_t wm[kR];
+#pragma unroll
+            for (int r = 0; r < kR; ++r)
+                wm[r] = __reduce_or_sync(kFull, (in_win && (pos >> 5) == (uint32_t)r) ? (1u << (pos & 31)) : 0u);
+            am = 0;
+            uint32_t wv[kR];
+#pragma unroll
+            for (int r = 0; r < kR; ++r) {
+                const uint32_t own = A_owner + __popc(wm[r] & lt_eq);
+                A_owner += __popc(wm[r]);
+                const uint32_t src = own & 31u;
+                const uint32_t ll = (ALG == ALG_BFS) ? level : __shfl_sync(kFull, A_lab, src);
+                const uint32_t x = A_x0 + 32u * r + lane;
+                const bool act = x < A_t.E;
+                am |= act ? (1u << r) : 0u;
+                u[r] = 0;
+                c[r] = ll;
+                wv[r] = 0;
+                if (SMP) {
+                    const uint32_t sd = __shfl_sync(kFull, A_t.sdelta, src);
+                    if (act) {
+                        u[r] = A_sbuf[sd + x];
+                        if (kW) wv[r] = A_sbuf[capw + sd + x];
+                    }
+                } else {
+                    const OffT dl = __shfl_sync(kFull, A_t.delta, src);
+                    if (act) {
+                        const OffT e = dl + (OffT)x;
+                        u[r] = ld_stream(&d.col[e], stream);
+                        if (kW) wv[r] = ld_stream(&d.w[e], stream);
+                    }
+                }
+            }
+            if (kW) {
+#pragma unroll
+                for (int r = 0; r < kR; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
+            }
+            // advance: next batch of this tile, or the next tile
+            A_x0 += 32u * kR;
+            if (A_x0 >= A_t.E) {
+                if (tn >= ntiles) {
+                    A_valid = false;
+                } else {
+                    A_t = nxt;
+                    ++kt;
+                    tn = next_tile();
+                    if (tn < ntiles) nxt = prepare(tn, (kt + 1) & 1);   // refills the stage of tile kt-1
+                    A_lab = (ALG == ALG_BFS) ? level : (A_t.sh.len ? ld_cg(&label[A_t.sh.v]) : 0u);
+                    A_x0 = 0;
+                    A_owner = 0xFFFFFFFFu;
+                    my_edges += A_t.E;
+                    if (SMP) {
+                        mbar_wait(&bars[kt & 1], (kt >> 1) & 1);
+                        __syncwarp();
+                        A_sbuf = wbuf + (size_t)(kt & 1) * kArrays * capw;
+                    }
+                }
+            }
+        };
+        // stage B: pre-filter gathers, then fire-and-forget commits
+        auto stage_b = [&](const uint32_t (&u)[kR], const uint32_t (&c)[kR], uint32_t am) {
+            if (d.tune & kTuneNoGather) {                     // replay experiment
+                uint32_t x = 0;
+#pragma unroll
+                for (int r = 0; r < kR; ++r) x += ((am >> r) & 1u) ? u[r] + c[r] : 0u;
+                if (x == 0x9E3779B9u) Q[0] = x;
+                return;
+            }
+            uint32_t cur[kR];
+            if (ALG == ALG_BFS) {
+                // visited test on the bitmap V (n/8 bytes, read-only in this
+                // kernel, cached in L1: hits never reach the L2 request path)
+#pragma unroll
+                for (int r = 0; r < kR; ++r)
+                    cur[r] = ((am >> r) & 1u) ? (((__ldg(&d.V[u[r] >> 5]) >> (u[r] & 31)) & 1u) ? 0u : kInf) : 0u;
+            } else {
+#pragma unroll
+                for (int r = 0; r < kR; ++r) cur[r] = ((am >> r) & 1u) ? ld_label(&filt[u[r]], keep) : 0u;
+            }
+            if (d.tune & kTuneNoCommit) {                     // replay experiment: count passes
+                uint32_t x = 0;
+#pragma unroll
+                for (int r = 0; r < kR; ++r) x += (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) ? 1u : 0u;
+                my_passes += x;
+                return;
+            }
+#pragma unroll
+            for (int r = 0; r < kR; ++r)
+                if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, markQ);
+        };
+        stage_a(u0, c0, am0);
+        for (;;) {
+            // two named register sets alternate, so no copies between iterations
+            const bool more1 = A_valid;
+            if (more1) stage_a(u1, c1, am1);
+            stage_b(u0, c0, am0);
+            if (!more1) break;
+            const bool more0 = A_valid;
+            if (more0) stage_a(u0, c0, am0);
+            stage_b(u1, c1, am1);
+            if (!more0) break;
+        }
+    }
+#else
     uint32_t t = next_tile();
     if (t < ntiles) {
         WarpTile<OffT, UDC> nxt = prepare(t, 0);
@@ -1114,8 +1275,14 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
             if (tn >= ntiles) break;
         }
     }
-    // statistics: one atomic per warp
-    if (lane == 0 && my_edges) atomicAdd(&ctl->edges, my_edges);
+#endif
+    // statistics: one global atomic per CTA (per-warp partials in shared memory)
+    __shared__ unsigned long long s_edges;
+    if (threadIdx.x == 0) s_edges = 0;
+    __syncthreads();
+    if (lane == 0 && my_edges) atomicAdd(&s_edges, my_edges);
+    __syncthreads();
+    if (threadIdx.x == 0 && s_edges) atomicAdd(&ctl->edges, s_edges);
     if (d.tune & kTuneNoCommit) {
         my_passes = __reduce_add_sync(kFull, my_passes);
         if (lane == 0 && my_passes) atomicAdd(&ctl->reached_v, (unsigned long long)my_passes);

@@ -15,13 +15,13 @@ from paper_conf_ipps_wangzlg19_b200 import dist as edist  # noqa: E402
 ALG = {"bfs": etg.BFS, "sssp": etg.SSSP, "cc": etg.CC, "sswp": etg.SSWP}
 
 
-def engines(g, P, K=32, flags=0):
+def engines(g, P, K=32, flags=0, sssp_delta=0):
     bounds = edist.partition_ranges(g.off, g.col, g.n, P)
     out = []
     for r in range(P):
         loff, lcol, lw = edist.partition_csr(g.off, g.col, g.w, g.n, bounds[r], bounds[r + 1])
         o, c, w, fl = etg.csr_to_device(loff, lcol, lw, device="cuda")
-        G = etg.Graph(o, c, w, n=g.n, K=K, flags=flags | fl, symmetric=g.symmetric)
+        G = etg.Graph(o, c, w, n=g.n, K=K, flags=flags | fl, symmetric=g.symmetric, sssp_delta=sssp_delta)
         out.append(edist.CudaEngine(G))
     return out
 
@@ -58,3 +58,14 @@ def test_partitioned_k_and_flags():
     for K, flags in ((8, 0), (1024, 0), (32, etg.NO_UDC)):
         labels, _ = edist.run_partitions(engines(g, 3, K, flags), edist.LoopbackGroup(), etg.SSSP, s)
         np.testing.assert_array_equal(etg.to_u32_numpy(labels), expected("sssp", g, s))
+
+
+@pytest.mark.parametrize("P", [1, 2, 3])
+@pytest.mark.parametrize("delta", [1, 16, 1 << 20])
+def test_partitioned_near_far_sssp(P, delta):
+    """The near-far SSSP schedule through the step-wise API: deferred vertices stay in the
+    exchanged bitmap, an empty near set re-scans with the next threshold."""
+    g = gg.make("C1")
+    s = gg.sample_sources(g, 1, 77 + P)[0]
+    labels, st = edist.run_partitions(engines(g, P, sssp_delta=delta), edist.LoopbackGroup(), etg.SSSP, s)
+    np.testing.assert_array_equal(etg.to_u32_numpy(labels), expected("sssp", g, s))
