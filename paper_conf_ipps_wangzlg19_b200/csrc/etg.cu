@@ -55,7 +55,8 @@ struct Params {
     bool warp;  // warp-centric expand (ts = 32, registers only); else the CTA-tile kernel
     bool idx;   // per-element owner index in shared memory (needs ts*K <= kCapE)
     bool smp;
-    bool prefetch;  // warp kernel: L2 bulk prefetch of the next tile's segments
+    bool prefetch;  // warp kernel: L2 bulk prefetch of the next tile's segments (ETG_TUNE 128)
+    bool ahead;     // warp kernel: next batch's segments loaded one batch ahead (SMP; off: ETG_NO_SMP)
     bool u64;
     uint32_t nf_delta;  // near-far SSSP bucket width (0 = paper schedule)
 };
@@ -79,6 +80,7 @@ Params derive(const etg_options *opt, uint32_t tune) {
     p.idx = p.udc && (uint64_t)p.ts * p.K <= kCapE;
     p.smp = p.idx && !(flags & ETG_NO_SMP);
     p.prefetch = false;
+    p.ahead = !(flags & ETG_NO_SMP);
     if (p.warp) {
         // warp kernel: tiles of 32 shadows; SMP = per-warp TMA stages of
         // 32 * (K + 6) words, affordable in shared memory for K <= 32
@@ -86,7 +88,10 @@ Params derive(const etg_options *opt, uint32_t tune) {
         p.idx = false;
         const bool host_edges = (flags & ETG_HOST_EDGES) != 0;   // no TMA on host-mapped memory
         p.smp = p.udc && (flags & ETG_SMP_SHARED) && !(flags & ETG_NO_SMP) && p.K <= 32 && !host_edges;
-        p.prefetch = p.udc && !(flags & ETG_NO_SMP) && !p.smp && !host_edges;
+        // the bulk prefetch is issued per lane through the uniform datapath (a
+        // 32-way serialised loop in SASS): measured slower than the register
+        // look-ahead alone, so it is an experiment switch only
+        p.prefetch = p.udc && (tune & 128u) && !(flags & ETG_NO_SMP) && !p.smp && !host_edges;
     }
     p.ts_log2 = 0;
     while ((1u << p.ts_log2) < p.ts) ++p.ts_log2;
@@ -94,7 +99,7 @@ Params derive(const etg_options *opt, uint32_t tune) {
 }
 
 struct Layout {
-    size_t Q, V, snap, F, B, D, S, tile_first, st_flag, st_agg, st_inc, ctl, total;
+    size_t Q, V, snap, F, B, D, S, tile_first, recE, recS, ctl, total;
     uint32_t nwords;
 };
 
@@ -120,9 +125,8 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
     L.D = take(4 * (n + 1));
     L.S = take(4 * (n + 2));
     L.tile_first = take(4 * max_tiles);
-    L.st_flag = take(4 * max_scan_tiles);
-    L.st_agg = take(8 * max_scan_tiles);
-    L.st_inc = take(8 * max_scan_tiles);
+    L.recE = take(8 * max_scan_tiles);
+    L.recS = take(8 * max_scan_tiles);
     L.ctl = take(sizeof(Ctl));
     L.total = o;
     return L;
@@ -173,13 +177,13 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.D = reinterpret_cast<uint32_t *>(g->ws + g->L.D);
     d.S = reinterpret_cast<uint32_t *>(g->ws + g->L.S);
     d.tile_first = reinterpret_cast<uint32_t *>(g->ws + g->L.tile_first);
-    d.st_flag = reinterpret_cast<uint32_t *>(g->ws + g->L.st_flag);
-    d.st_agg = reinterpret_cast<unsigned long long *>(g->ws + g->L.st_agg);
-    d.st_inc = reinterpret_cast<unsigned long long *>(g->ws + g->L.st_inc);
+    d.recE = reinterpret_cast<unsigned long long *>(g->ws + g->L.recE);
+    d.recS = reinterpret_cast<unsigned long long *>(g->ws + g->L.recS);
     d.ctl = g->ctl;
     d.n = (uint32_t)g->n;
     d.m = g->m;
     d.prefetch = g->p.prefetch ? 1u : 0u;
+    d.ahead = g->p.ahead ? 1u : 0u;
     d.K = g->p.K;
     d.ts = g->p.ts;
     d.ts_log2 = g->p.ts_log2;
@@ -643,7 +647,7 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
         (e = cudaEventCreate(&g->pev[2])) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), g->stream)) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ws + L.Q, 0, 4ull * L.nwords, g->stream)) != cudaSuccess ||
-        (e = cudaMemsetAsync(g->ws + L.st_flag, 0, L.st_agg - L.st_flag, g->stream)) != cudaSuccess) {
+        (e = cudaMemsetAsync(g->ws + L.recE, 0, L.ctl - L.recE, g->stream)) != cudaSuccess) {
         return bail(fail(ETG_ECUDA, std::string("load: ") + cudaGetErrorString(e)));
     }
     g->tune = tune;

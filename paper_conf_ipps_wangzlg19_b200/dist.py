@@ -9,12 +9,16 @@ Design:
   (global ids) -- relaxations on rank g only ever touch owned vertices;
 * every rank expands the same, replicated, compacted active set (UDC over its
   own sub-rows, so a hub's edges are split ~deg/P per rank), marks improved
-  owned vertices in its bitmap, then the exchange makes the bitmaps the union
-  (ranges are word-disjoint, so an integer all-reduce SUM is the OR) and, for
-  SSSP/CC/SSWP, the labels the element-wise best (MIN; MAX for SSWP): a
-  non-owner's copy is the owner's value from an earlier exchange, never better
-  than the owner's current one.  BFS exchanges the bitmap only -- each rank's
-  scan writes the depth of every vertex of the new active set.
+  owned vertices in its bitmap (BFS, near-far SSSP), then the exchange makes
+  the bitmaps the union and, for SSSP/CC/SSWP, the labels the element-wise best
+  (MIN; MAX for SSWP): a non-owner's copy is the owner's value from an earlier
+  exchange, never better than the owner's current one.  Union = unsigned MAX
+  per word: a word's new bits come from its owner only, and the bits every
+  rank holds already (near-far's deferred vertices) are the same on all ranks,
+  so the owner's word is a superset of every other rank's.  SSSP/CC/SSWP mark
+  nothing otherwise: each rank's scan activates the vertices whose (exchanged)
+  label moved.  BFS exchanges the bitmap only -- each rank's scan writes the
+  depth of every vertex of the new active set.
 * termination: the number of activated vertices (bitmap bits consumed by the
   scan) is identical on every rank after the exchange, so all ranks leave the
   loop together (the compacted sizes differ: they count local out-edges).
@@ -156,7 +160,12 @@ class CudaEngine:
 
 def _exchange(engines, group, alg: int) -> None:
     """Union of the bitmaps; best labels (SSSP/CC: min, SSWP: max) -- see module doc."""
-    group.allreduce([e.q for e in engines], "sum")
+    qs = [e.q for e in engines]
+    for t in qs:
+        t.bitwise_xor_(SIGN)                # uint32 order -> int32 order
+    group.allreduce(qs, "max")              # superset words: unsigned MAX = OR
+    for t in qs:
+        t.bitwise_xor_(SIGN)
     if alg != BFS:
         labs = [e.labels for e in engines]
         for t in labs:

@@ -124,17 +124,19 @@ def test_k_invariance(c1, c1sym, K):
 
 @pytest.mark.parametrize("flags", [2, 4, 32, 2 | 32, 4 | 32, 128, 128 | 32])
 def test_flag_invariance(c1, c1sym, flags):
-    """UDC off (L88 baseline), SMP off (Fig. 6 ablation), shared-memory SMP, host-driven loop."""
+    """UDC off (L88 baseline), SMP off (Fig. 6 ablation: no look-ahead), shared-memory SMP,
+    host-driven loop."""
     srcs = gg.sample_sources(c1, 2, 5)
     check_all(c1, srcs, flags=flags)
     check_cc(c1sym, flags=flags)
 
 
-@pytest.mark.parametrize("tune", [64, 2, 2 | 64])
+@pytest.mark.parametrize("tune", [64, 2, 2 | 64, 128])
 def test_engine_variants(c1, c1sym, monkeypatch, tune):
     """Engine variants picked at load time (ETG_TUNE): 64 = SSSP/CC/SSWP commits mark the
     bitmap and the scan reads only it (no label/snapshot comparison);
-    2 = the CTA-tile expand kernel.  Labels are the same unique fixpoints."""
+    2 = the CTA-tile expand kernel; 128 = L2 bulk prefetch of the next tile's segments.
+    Labels are the same unique fixpoints."""
     monkeypatch.setenv("ETG_TUNE", str(tune))
     srcs = gg.sample_sources(c1, 2, 17)
     check_all(c1, srcs)
