@@ -46,7 +46,7 @@ constexpr uint32_t kFull = 0xFFFFFFFFu;
 #define ETG_KR 8
 #endif
 #ifndef ETG_MINB
-#define ETG_MINB 1
+#define ETG_MINB 3                          // expand: >= 3 CTAs (24 warps) per SM, <= 85 registers
 #endif
 #ifndef ETG_PIPE
 #define ETG_PIPE 1                          // software-pipelined batch loop in the warp expand
@@ -93,9 +93,8 @@ struct Dev {
     uint32_t *D;                // out-degree of F[k] (> 0)
     uint32_t *S;                // exclusive prefix of shadow counts (nF + 1 entries)
     uint32_t *tile_first;       // entry owning shadow t*ts
-    uint32_t *st_flag;          // chained scan: per scan tile (epoch << 2 | flag)
-    unsigned long long *st_agg; //   aggregate  (entries << 32 | shadows)
-    unsigned long long *st_inc; //   inclusive prefix, same packing
+    unsigned long long *recE;   // chained scan records per scan tile: kept entries
+    unsigned long long *recS;   //   and shadows (value << 32 | epoch << 2 | flag)
     Ctl *ctl;
     unsigned long long m;       // edges
     uint32_t n;
@@ -105,6 +104,7 @@ struct Dev {
     uint32_t ts_log2;
     uint32_t tune;              // experiment switches (ETG_TUNE env var at load); 0 = default
     uint32_t prefetch;          // warp kernel, direct mode: L2 bulk prefetch of the next tile
+    uint32_t ahead;             // warp kernel: stage A of the next batch before stage B of this one
     uint32_t nf_delta;          // near-far SSSP bucket width (0: the paper's schedule)
 };
 
@@ -113,6 +113,7 @@ constexpr uint32_t kTuneFilterL1 = 1u;    // pre-filter label loads cached in L1
 constexpr uint32_t kTuneNoGather = 16u;   // skip the label gather and the commit
 constexpr uint32_t kTuneNoCommit = 32u;   // gather labels but never commit (counts passes)
 constexpr uint32_t kTuneQMark = 64u;      // A/B: SSSP/CC/SSWP commits also set Q, the scan reads only Q
+constexpr uint32_t kTuneScanDyn = 256u;   // A/B: every scan tile from the counter (no static first tile)
 
 // ------------------------------------------------------------------------- //
 // small device helpers
@@ -327,6 +328,48 @@ constexpr int kG = 8;                                     // words whose loads a
 constexpr uint32_t kScanV = (uint32_t)kWarps * kWPW * 32; // vertices per scan tile (8192)
 constexpr int kLB = 4;                                    // look-back window: 32 * kLB predecessor tiles
 
+__device__ __forceinline__ void st_volatile_u64(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.volatile.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
+}
+
+// One look-back window (see udc_scan_kernel): records r[k] of tiles p - lane -
+// 32k.  Waits (returns without progress) while a needed predecessor has not
+// published; else adds the values up to and including the nearest inclusive
+// prefix (done) or the whole window (moves p back by the window).
+template <int N>
+__device__ __forceinline__ void lookback_resolve(const unsigned long long (&r)[N], uint32_t eb, int &p,
+                                                 uint32_t &excl, bool &done) {
+    const uint32_t lane = lane_id();
+    int firstk = N;
+    uint32_t first = 32;
+    bool wait = false;
+#pragma unroll
+    for (int k = 0; k < N; ++k) {
+        const uint32_t lo = (uint32_t)r[k];
+        const bool valid = (lo & ~3u) == eb && (lo & 3u) != 0;
+        const uint32_t incl = __ballot_sync(kFull, valid && (lo & 3u) == 2u);
+        const uint32_t inval = __ballot_sync(kFull, !valid);
+        if (firstk == N) {
+            if (incl) {
+                firstk = k;
+                first = (uint32_t)(__ffs(incl) - 1);
+                const uint32_t need = first < 31 ? ((2u << first) - 1u) : kFull;
+                if (inval & need) wait = true;
+            } else if (inval) {
+                wait = true;
+            }
+        }
+    }
+    if (wait) return;
+    uint32_t v = 0;
+#pragma unroll
+    for (int k = 0; k < N; ++k)
+        if (k < firstk || (k == firstk && lane <= first)) v += (uint32_t)(r[k] >> 32);
+    excl += __reduce_add_sync(kFull, v);
+    if (firstk < N) done = true;
+    else p -= 32 * N;
+}
+
 template <class OffT, bool UDC, bool BFSLAB>
 __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraphConditionalHandle cond,
                                                           int use_cond) {
@@ -346,11 +389,17 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
     const uint32_t new_depth = ctl->depth + 1;            // BFS depth of the vertices in Q
     const uint32_t th = ctl->thresh;                      // near-far threshold (SSSP option)
     const bool qmark = !d.nf_delta && (d.tune & kTuneQMark);   // A/B switch: the expand marks Q itself
-    for (;;) {
-        if (threadIdx.x == 0) s_tile = atomicAdd(&ctl->scan_ctr, 1u);
-        __syncwarp();
-        __syncthreads();
-        const uint32_t tile = s_tile;
+    const bool stat = !(d.tune & kTuneScanDyn);
+    for (uint32_t round = 0;; ++round) {
+        // first tile = blockIdx.x (CTAs are dispatched in index order, so a
+        // tile's predecessors are resident); later tiles from a counter
+        if (round > 0 || !stat) {
+            if (stat && gridDim.x >= nscan) break;        // every tile was taken in round 0
+            if (threadIdx.x == 0) s_tile = (stat ? gridDim.x : 0u) + atomicAdd(&ctl->scan_ctr, 1u);
+            __syncwarp();
+            __syncthreads();
+        }
+        const uint32_t tile = (round == 0 && stat) ? blockIdx.x : s_tile;
         __syncthreads();                                  // all have read s_tile before it is reused
         if (tile >= nscan) break;
         const uint32_t wbase = (tile * kWarps + warp) * kWPW;          // first word of this warp
@@ -475,74 +524,41 @@ __global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraph
             btotal += x;
         }
         if (threadIdx.x < 32) {
-            u64 excl = 0;
-            if (tile == 0) {
-                if (lane == 0) {
-                    d.st_inc[0] = btotal;
-                    __threadfence();
-                    atomicExch(&d.st_flag[0], (epoch << 2) | 2u);
-                }
-            } else {
-                if (lane == 0) {
-                    d.st_agg[tile] = btotal;
-                    __threadfence();
-                    atomicExch(&d.st_flag[tile], (epoch << 2) | 1u);
-                }
-                // Window of 32 * kLB predecessors, all flag loads in flight at
-                // once: position i = 32k + lane is tile p - i.  Aggregates are
-                // published before any look-back, so a tile sums them directly
-                // up to the nearest inclusive prefix without waiting for its
-                // neighbours' look-backs (one round trip for <= 32 * kLB tiles).
-                int p = (int)tile - 1;                  // nearest predecessor at position 0
-                for (;;) {
-                    uint32_t f[kLB];
+            // Single-pass chained scan, one 64-bit record per tile and per
+            // quantity (E = kept entries, S = shadows): value << 32 | epoch << 2
+            // | flag (1 aggregate, 2 inclusive prefix).  A record is one aligned
+            // 64-bit store, so value and flag are seen together (no fences).
+            // Look-back: a window of 32 * kLB predecessors, all loads in flight
+            // at once; aggregates are summed up to the nearest inclusive prefix.
+            const uint32_t eb = epoch << 2;
+            const uint32_t aggE = (uint32_t)(btotal >> 32), aggS = (uint32_t)btotal;
+            uint32_t exclE = 0, exclS = 0;
+            if (lane == 0) {
+                const uint32_t fl = tile == 0 ? 2u : 1u;
+                st_volatile_u64(&d.recE[tile], ((u64)aggE << 32) | eb | fl);
+                st_volatile_u64(&d.recS[tile], ((u64)aggS << 32) | eb | fl);
+            }
+            if (tile > 0) {
+                bool doneE = false, doneS = false;
+                int pE = (int)tile - 1, pS = (int)tile - 1;   // nearest predecessor at window position 0
+                const u64 none = (u64)(eb | 1u);               // beyond tile 0: an empty aggregate
+                while (!(doneE && doneS)) {
+                    u64 re[kLB], rs[kLB];
 #pragma unroll
                     for (int k = 0; k < kLB; ++k) {
-                        const int q = p - (int)lane - 32 * k;
-                        f[k] = (epoch << 2) | 1u;       // q < 0: beyond tile 0, contributes 0
-                        if (q >= 0) f[k] = ld_volatile_u32(&d.st_flag[q]);
+                        const int qE = pE - (int)lane - 32 * k, qS = pS - (int)lane - 32 * k;
+                        re[k] = (doneE || qE < 0) ? none : ld_volatile_u64(&d.recE[qE]);
+                        rs[k] = (doneS || qS < 0) ? none : ld_volatile_u64(&d.recS[qS]);
                     }
-                    int firstk = kLB;                   // window row of the nearest inclusive prefix
-                    uint32_t first = 32;                //   and its lane
-                    bool wait = false;
-#pragma unroll
-                    for (int k = 0; k < kLB; ++k) {
-                        const int q = p - (int)lane - 32 * k;
-                        const bool valid = (f[k] >> 2) == epoch && (f[k] & 3u) != 0;
-                        const uint32_t incl = __ballot_sync(kFull, valid && (f[k] & 3u) == 2u && q >= 0);
-                        const uint32_t inval = __ballot_sync(kFull, !valid);
-                        if (firstk == kLB) {
-                            if (incl) {
-                                firstk = k;
-                                first = (uint32_t)(__ffs(incl) - 1);
-                                const uint32_t need = first < 31 ? ((2u << first) - 1u) : kFull;
-                                if (inval & need) wait = true;
-                            } else if (inval) {
-                                wait = true;
-                            }
-                        }
-                    }
-                    if (wait) continue;                 // a needed predecessor is not published yet
-                    __threadfence();
-                    u64 val = 0;
-#pragma unroll
-                    for (int k = 0; k < kLB; ++k) {
-                        const int q = p - (int)lane - 32 * k;
-                        if (q < 0) continue;
-                        if (k < firstk || (k == firstk && lane < first)) val += ld_volatile_u64(&d.st_agg[q]);
-                        else if (k == firstk && lane == first) val += ld_volatile_u64(&d.st_inc[q]);
-                    }
-                    excl += warp_sum_u64(val);
-                    if (firstk < kLB) break;
-                    p -= 32 * kLB;
+                    if (!doneE) lookback_resolve(re, eb, pE, exclE, doneE);
+                    if (!doneS) lookback_resolve(rs, eb, pS, exclS, doneS);
                 }
                 if (lane == 0) {
-                    d.st_inc[tile] = excl + btotal;
-                    __threadfence();
-                    atomicExch(&d.st_flag[tile], (epoch << 2) | 2u);
+                    st_volatile_u64(&d.recE[tile], ((u64)(exclE + aggE) << 32) | eb | 2u);
+                    st_volatile_u64(&d.recS[tile], ((u64)(exclS + aggS) << 32) | eb | 2u);
                 }
             }
-            if (lane == 0) s_prefix = excl;
+            if (lane == 0) s_prefix = ((u64)exclE << 32) | exclS;
             __syncwarp();
         }
         __syncthreads();
@@ -1173,7 +1189,15 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
                 if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, markQ);
         };
         stage_a(u0, c0, am0);
-        for (;;) {
+        if (!d.ahead) {
+            // ETG_NO_SMP ("w/o SMP" ablation): each batch's segments are loaded
+            // and relaxed back to back, nothing is fetched ahead of its use
+            for (;;) {
+                stage_b(u0, c0, am0);
+                if (!A_valid) break;
+                stage_a(u0, c0, am0);
+            }
+        } else for (;;) {
             // two named register sets alternate, so no copies between iterations
             const bool more1 = A_valid;
             if (more1) stage_a(u1, c1, am1);
