@@ -48,10 +48,16 @@ constexpr uint32_t kFull = 0xFFFFFFFFu;
 #ifndef ETG_MINB
 #define ETG_MINB 3                          // expand: >= 3 CTAs (24 warps) per SM, <= 85 registers
 #endif
+#ifndef ETG_SGRAB
+#define ETG_SGRAB 1                         // expand: first tile grab static (global warp index)
+#endif
 #ifndef ETG_PIPE
 #define ETG_PIPE 1                          // software-pipelined batch loop in the warp expand
 #endif
 constexpr int kR = ETG_KR;                  // edges (chunks) in flight per thread in the relax loop
+#ifndef ETG_KR_W
+#define ETG_KR_W 6                          // ... for SSSP/SSWP (weights: two streams per chunk)
+#endif
 
 enum Alg : int { ALG_BFS = 0, ALG_SSSP = 1, ALG_CC = 2, ALG_SSWP = 3 };
 
@@ -958,6 +964,7 @@ template <class OffT, int ALG, bool UDC, bool SMP>
 __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT> d, uint32_t capw) {
     constexpr bool kW = (ALG == ALG_SSSP || ALG == ALG_SSWP);
     constexpr uint32_t kArrays = kW ? 2u : 1u;
+    constexpr int kRB = kW ? ETG_KR_W : kR;                // chunks per batch (weighted: fewer, no spills)
     extern __shared__ __align__(128) uint8_t dyn_smem[];
     Ctl *ctl = d.ctl;
     const uint32_t nF = ctl->nF, N = ctl->nshadow, ntiles = ctl->ntiles;
@@ -998,13 +1005,25 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
 
     // Dynamic schedule: a warp grabs kGrab consecutive tiles at a time, so the
     // slowest warp ends within one grab of the rest (tiles carry 32..32K edges).
+    // The first grab is static (global warp index), later ones come from the
+    // counter: a small active set costs no atomic at all, and a large one
+    // one atomic per grab after the first.
     constexpr uint32_t kGrab = 2;
+    const uint32_t n_static = gridDim.x * kWarps * kGrab;
     uint32_t g_next = 0, g_end = 0;
+    bool first_grab = true;
     auto next_tile = [&]() -> uint32_t {
         if (g_next == g_end) {
             uint32_t g = 0;
-            if (lane == 0) g = atomicAdd(&ctl->tile_ctr, kGrab);
-            g_next = __shfl_sync(kFull, g, 0);
+            if (first_grab && ETG_SGRAB) {
+                g = (blockIdx.x * kWarps + wib) * kGrab;
+                first_grab = false;
+            } else {
+                const uint32_t base = ETG_SGRAB ? n_static : 0u;
+                if (lane == 0 && base < ntiles) g = base + atomicAdd(&ctl->tile_ctr, kGrab);
+                g = base < ntiles ? __shfl_sync(kFull, g, 0) : ntiles;
+            }
+            g_next = g;
             g_end = g_next >= ntiles ? g_next : min(g_next + kGrab, ntiles);
             if (g_next >= ntiles) return ntiles;
         }
@@ -1065,7 +1084,7 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
     };
 
 #if ETG_PIPE
-    // Software pipeline over the warp's stream of batches (kR chunks of 32
+    // Software pipeline over the warp's stream of batches (kRB chunks of 32
     // elements; a tile is one or more batches).  Stage A of batch b+1 (owner
     // masks, column/weight loads, candidates) is issued before stage B of batch
     // b (label gathers, commits), so the column loads of the next batch are in
@@ -1092,20 +1111,20 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
         }
         my_edges += A_t.E;
         bool A_valid = true;
-        uint32_t u0[kR], c0[kR], u1[kR], c1[kR];
+        uint32_t u0[kRB], c0[kRB], u1[kRB], c1[kRB];
         uint32_t am0 = 0, am1 = 0;
         // stage A: the batch at (A_t, A_x0) into (u, c, am); then advance the cursor
-        auto stage_a = [&](uint32_t (&u)[kR], uint32_t (&c)[kR], uint32_t &am) {
+        auto stage_a = [&](uint32_t (&u)[kRB], uint32_t (&c)[kRB], uint32_t &am) {
             const uint32_t pos = A_t.o - A_x0;                 // this lane's slice start in the batch
-            const bool in_win = A_t.sh.len && pos < 32u * kR;
-            uint32_t wm[kR];
+            const bool in_win = A_t.sh.len && pos < 32u * kRB;
+            uint32_t wm[kRB];
 #pragma unroll
-            for (int r = 0; r < kR; ++r)
+            for (int r = 0; r < kRB; ++r)
                 wm[r] = __reduce_or_sync(kFull, (in_win && (pos >> 5) == (uint32_t)r) ? (1u << (pos & 31)) : 0u);
             am = 0;
-            uint32_t wv[kR];
+            uint32_t wv[kRB];
 #pragma unroll
-            for (int r = 0; r < kR; ++r) {
+            for (int r = 0; r < kRB; ++r) {
                 const uint32_t own = A_owner + __popc(wm[r] & lt_eq);
                 A_owner += __popc(wm[r]);
                 const uint32_t src = own & 31u;
@@ -1133,10 +1152,10 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
             }
             if (kW) {
 #pragma unroll
-                for (int r = 0; r < kR; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
+                for (int r = 0; r < kRB; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
             }
             // advance: next batch of this tile, or the next tile
-            A_x0 += 32u * kR;
+            A_x0 += 32u * kRB;
             if (A_x0 >= A_t.E) {
                 if (tn >= ntiles) {
                     A_valid = false;
@@ -1158,34 +1177,34 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
             }
         };
         // stage B: pre-filter gathers, then fire-and-forget commits
-        auto stage_b = [&](const uint32_t (&u)[kR], const uint32_t (&c)[kR], uint32_t am) {
+        auto stage_b = [&](const uint32_t (&u)[kRB], const uint32_t (&c)[kRB], uint32_t am) {
             if (d.tune & kTuneNoGather) {                     // replay experiment
                 uint32_t x = 0;
 #pragma unroll
-                for (int r = 0; r < kR; ++r) x += ((am >> r) & 1u) ? u[r] + c[r] : 0u;
+                for (int r = 0; r < kRB; ++r) x += ((am >> r) & 1u) ? u[r] + c[r] : 0u;
                 if (x == 0x9E3779B9u) Q[0] = x;
                 return;
             }
-            uint32_t cur[kR];
+            uint32_t cur[kRB];
             if (ALG == ALG_BFS) {
                 // visited test on the bitmap V (n/8 bytes, read-only in this
                 // kernel, cached in L1: hits never reach the L2 request path)
 #pragma unroll
-                for (int r = 0; r < kR; ++r)
+                for (int r = 0; r < kRB; ++r)
                     cur[r] = ((am >> r) & 1u) ? (((__ldg(&d.V[u[r] >> 5]) >> (u[r] & 31)) & 1u) ? 0u : kInf) : 0u;
             } else {
 #pragma unroll
-                for (int r = 0; r < kR; ++r) cur[r] = ((am >> r) & 1u) ? ld_label(&filt[u[r]], keep) : 0u;
+                for (int r = 0; r < kRB; ++r) cur[r] = ((am >> r) & 1u) ? ld_label(&filt[u[r]], keep) : 0u;
             }
             if (d.tune & kTuneNoCommit) {                     // replay experiment: count passes
                 uint32_t x = 0;
 #pragma unroll
-                for (int r = 0; r < kR; ++r) x += (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) ? 1u : 0u;
+                for (int r = 0; r < kRB; ++r) x += (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) ? 1u : 0u;
                 my_passes += x;
                 return;
             }
 #pragma unroll
-            for (int r = 0; r < kR; ++r)
+            for (int r = 0; r < kRB; ++r)
                 if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, markQ);
         };
         stage_a(u0, c0, am0);
@@ -1229,21 +1248,21 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
                 sbuf = wbuf + (size_t)(k & 1) * kArrays * capw;
             }
             uint32_t owner = 0xFFFFFFFFu;                     // owner of the element before x0
-            // Batches of kR chunks of 32 elements.  The owner of element x is
-            // the number of slice starts <= x, minus one: the batch's kR words of
-            // the start mask come from kR independent OR-reductions, then a
+            // Batches of kRB chunks of 32 elements.  The owner of element x is
+            // the number of slice starts <= x, minus one: the batch's kRB words of
+            // the start mask come from kRB independent OR-reductions, then a
             // popcount prefix -- no serial dependency between chunks.
-            for (uint32_t x0 = 0; x0 < E; x0 += 32u * kR) {
-                uint32_t u[kR], c[kR], cur[kR], wv[kR];
-                bool act[kR];
+            for (uint32_t x0 = 0; x0 < E; x0 += 32u * kRB) {
+                uint32_t u[kRB], c[kRB], cur[kRB], wv[kRB];
+                bool act[kRB];
                 const uint32_t pos = o - x0;                  // this lane's slice start in the batch
-                const bool in_win = sh.len && pos < 32u * kR;
-                uint32_t wm[kR];
+                const bool in_win = sh.len && pos < 32u * kRB;
+                uint32_t wm[kRB];
 #pragma unroll
-                for (int r = 0; r < kR; ++r)
+                for (int r = 0; r < kRB; ++r)
                     wm[r] = __reduce_or_sync(kFull, (in_win && (pos >> 5) == (uint32_t)r) ? (1u << (pos & 31)) : 0u);
 #pragma unroll
-                for (int r = 0; r < kR; ++r) {
+                for (int r = 0; r < kRB; ++r) {
                     const uint32_t own = owner + __popc(wm[r] & lt_eq);
                     owner += __popc(wm[r]);
                     const uint32_t src = own & 31u;
@@ -1270,12 +1289,12 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
                 }
                 if (kW) {
 #pragma unroll
-                    for (int r = 0; r < kR; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
+                    for (int r = 0; r < kRB; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
                 }
                 if (d.tune & kTuneNoGather) {                 // replay experiment
                     uint32_t x = 0;
 #pragma unroll
-                    for (int r = 0; r < kR; ++r) x += act[r] ? u[r] + c[r] : 0u;
+                    for (int r = 0; r < kRB; ++r) x += act[r] ? u[r] + c[r] : 0u;
                     if (x == 0x9E3779B9u) Q[0] = x;
                     continue;
                 }
@@ -1284,16 +1303,16 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
                 // and the red.min/max commits never touch the same lines (R-4, R-6)
                 const uint32_t *filt = (ALG == ALG_BFS) ? label : d.snap;
 #pragma unroll
-                for (int r = 0; r < kR; ++r) cur[r] = act[r] ? ld_label(&filt[u[r]], keep) : 0u;
+                for (int r = 0; r < kRB; ++r) cur[r] = act[r] ? ld_label(&filt[u[r]], keep) : 0u;
                 if (d.tune & kTuneNoCommit) {                 // replay experiment: count passes
                     uint32_t x = 0;
 #pragma unroll
-                    for (int r = 0; r < kR; ++r) x += (act[r] && improves<ALG>(c[r], cur[r])) ? 1u : 0u;
+                    for (int r = 0; r < kRB; ++r) x += (act[r] && improves<ALG>(c[r], cur[r])) ? 1u : 0u;
                     my_passes += x;
                     continue;
                 }
 #pragma unroll
-                for (int r = 0; r < kR; ++r)
+                for (int r = 0; r < kRB; ++r)
                     if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, d.nf_delta != 0 || (d.tune & kTuneQMark));
             }
             if (tn >= ntiles) break;
