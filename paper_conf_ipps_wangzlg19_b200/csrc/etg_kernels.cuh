@@ -377,7 +377,7 @@ __device__ __forceinline__ void lookback_resolve(const unsigned long long (&r)[N
 }
 
 template <class OffT, bool UDC, bool BFSLAB>
-__global__ __launch_bounds__(kBlock) void udc_scan_kernel(Dev<OffT> d, cudaGraphConditionalHandle cond,
+__global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGraphConditionalHandle cond,
                                                           int use_cond) {
     typedef unsigned long long u64;
     __shared__ uint32_t s_tile;
@@ -1192,6 +1192,11 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
 #pragma unroll
                 for (int r = 0; r < kRB; ++r)
                     cur[r] = ((am >> r) & 1u) ? (((__ldg(&d.V[u[r] >> 5]) >> (u[r] & 31)) & 1u) ? 0u : kInf) : 0u;
+            } else if (ALG == ALG_CC && level == 1) {
+                // CC's first expand: the snapshot is still the initial labelling
+                // label[u] = u (A1), so the pre-filter needs no gather at all
+#pragma unroll
+                for (int r = 0; r < kRB; ++r) cur[r] = u[r];
             } else {
 #pragma unroll
                 for (int r = 0; r < kRB; ++r) cur[r] = ((am >> r) & 1u) ? ld_label(&filt[u[r]], keep) : 0u;
