@@ -330,7 +330,10 @@ __global__ __launch_bounds__(kBlock) void init_kernel(Dev<OffT> d, uint32_t *lab
 #define ETG_WPW 32
 #endif
 constexpr int kWPW = ETG_WPW;                             // bitmap words per warp per tile
-constexpr int kG = 8;                                     // words whose loads are in flight together
+#ifndef ETG_SCAN_G
+#define ETG_SCAN_G 8
+#endif
+constexpr int kG = ETG_SCAN_G;                            // words whose loads are in flight together
 constexpr uint32_t kScanV = (uint32_t)kWarps * kWPW * 32; // vertices per scan tile (8192)
 constexpr int kLB = 4;                                    // look-back window: 32 * kLB predecessor tiles
 
@@ -544,7 +547,10 @@ __global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGr
                 st_volatile_u64(&d.recE[tile], ((u64)aggE << 32) | eb | fl);
                 st_volatile_u64(&d.recS[tile], ((u64)aggS << 32) | eb | fl);
             }
-            if (tile > 0) {
+            // A tile with nothing to write needs no prefix: its aggregate (0)
+            // lets successors look past it.  Only the last tile, which
+            // publishes the totals, always resolves its prefix.
+            if (tile > 0 && (btotal != 0 || tile == nscan - 1)) {
                 bool doneE = false, doneS = false;
                 int pE = (int)tile - 1, pS = (int)tile - 1;   // nearest predecessor at window position 0
                 const u64 none = (u64)(eb | 1u);               // beyond tile 0: an empty aggregate

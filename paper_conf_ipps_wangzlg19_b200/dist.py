@@ -19,6 +19,9 @@ Design:
   nothing otherwise: each rank's scan activates the vertices whose (exchanged)
   label moved.  BFS exchanges the bitmap only -- each rank's scan writes the
   depth of every vertex of the new active set.
+* collective: an all-gather of the owned slices (bitmap words, labels) -- see
+  ``_exchange``; a full-array all-reduce (MAX on the bitmap, MIN/MAX on the
+  labels) is kept as the fallback without partition bounds;
 * termination: the number of activated vertices (bitmap bits consumed by the
   scan) is identical on every rank after the exchange, so all ranks leave the
   loop together (the compacted sizes differ: they count local out-edges).
@@ -94,7 +97,7 @@ def partition_csr(off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor
 # collectives
 # --------------------------------------------------------------------------- #
 class TorchDistGroup:
-    """all_reduce over a torch.distributed process group (NCCL on GPUs, gloo on CPUs)."""
+    """Collectives over a torch.distributed process group (NCCL on GPUs, gloo on CPUs)."""
 
     def __init__(self, group=None):
         import torch.distributed as dist
@@ -106,6 +109,23 @@ class TorchDistGroup:
                "max": self.dist.ReduceOp.MAX}
         assert len(tensors) == 1
         self.dist.all_reduce(tensors[0], op=ops[op], group=self.group)
+
+    def allgather_ranges(self, tensors: Sequence[torch.Tensor], bounds: Sequence[int]) -> None:
+        """Rank r's slice [bounds[r], bounds[r+1]) of its tensor is authoritative:
+        after the call every rank's tensor holds every rank's slice (one
+        all-gather of equal-sized, padded slices)."""
+        assert len(tensors) == 1
+        t = tensors[0]
+        r = self.dist.get_rank(self.group)
+        P = len(bounds) - 1
+        width = max(bounds[q + 1] - bounds[q] for q in range(P))
+        send = torch.zeros(width, dtype=t.dtype, device=t.device)
+        send[:bounds[r + 1] - bounds[r]] = t[bounds[r]:bounds[r + 1]]
+        recv = [torch.empty_like(send) for _ in range(P)]
+        self.dist.all_gather(recv, send, group=self.group)
+        for q in range(P):
+            if q != r:
+                t[bounds[q]:bounds[q + 1]] = recv[q][:bounds[q + 1] - bounds[q]]
 
 
 class LoopbackGroup:
@@ -122,6 +142,12 @@ class LoopbackGroup:
                 acc = torch.maximum(acc, t)
         for t in tensors:
             t.copy_(acc)
+
+    def allgather_ranges(self, tensors: Sequence[torch.Tensor], bounds: Sequence[int]) -> None:
+        for q, src in enumerate(tensors):
+            for t in tensors:
+                if t is not src:
+                    t[bounds[q]:bounds[q + 1]] = src[bounds[q]:bounds[q + 1]]
 
 
 # --------------------------------------------------------------------------- #
@@ -158,8 +184,20 @@ class CudaEngine:
         return st
 
 
-def _exchange(engines, group, alg: int) -> None:
-    """Union of the bitmaps; best labels (SSSP/CC: min, SSWP: max) -- see module doc."""
+def _exchange(engines, group, alg: int, bounds: Optional[Sequence[int]] = None) -> None:
+    """Union of the bitmaps; best labels (SSSP/CC: min, SSWP: max) -- see module doc.
+
+    With the partition bounds: an all-gather of every rank's OWNED slices (its
+    bitmap words and, for SSSP/CC/SSWP, its labels).  Relaxations only ever
+    touch owned vertices, so the owner's slice already is the union / the
+    best value, and each rank sends n/32 words / P (+ n labels / P) instead of
+    reducing full-size arrays.  Without bounds: full-size all-reduces."""
+    if bounds is not None:
+        wb = [(b + 31) // 32 for b in bounds]          # boundaries are multiples of 32 (last: n)
+        group.allgather_ranges([e.q for e in engines], wb)
+        if alg != BFS:
+            group.allgather_ranges([e.labels for e in engines], bounds)
+        return
     qs = [e.q for e in engines]
     for t in qs:
         t.bitwise_xor_(SIGN)                # uint32 order -> int32 order
@@ -175,15 +213,17 @@ def _exchange(engines, group, alg: int) -> None:
             t.bitwise_xor_(SIGN)
 
 
-def run_partitions(engines, group, alg: int, source: int = 0):
+def run_partitions(engines, group, alg: int, source: int = 0, bounds: Optional[Sequence[int]] = None):
     """Drive P engines in lockstep (all in this process: loopback), or ONE
     engine of this rank (torch.distributed: the other ranks run the same
-    loop).  Returns (labels of engines[0], summed stats, iterations)."""
+    loop).  ``bounds`` (the partition, ``partition_ranges``) selects the
+    all-gather exchange of owned slices; without it full arrays are
+    all-reduced.  Returns (labels of engines[0], summed stats)."""
     n_act = [e.begin(alg, source) for e in engines]
     while n_act[0] > 0:
         for e in engines:
             e.expand()
-        _exchange(engines, group, alg)
+        _exchange(engines, group, alg, bounds)
         n_act = [e.scan() for e in engines]
         if len(set(n_act)) != 1:
             raise EtgError(f"ranks disagree on the active-set size: {n_act}")
@@ -211,4 +251,4 @@ class DistGraph:
         self.group = TorchDistGroup(group)
 
     def run(self, alg: int, source: int = 0):
-        return run_partitions([self.engine], self.group, alg, source)
+        return run_partitions([self.engine], self.group, alg, source, self.bounds)

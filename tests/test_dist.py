@@ -61,19 +61,22 @@ def test_partition_properties(P):
     assert seen == g.m
 
 
+@pytest.mark.parametrize("gather", [False, True])
 @pytest.mark.parametrize("alg", ["bfs", "sssp", "cc", "sswp"])
 @pytest.mark.parametrize("P", [2, 3])
-def test_loopback_driver_matches_oracle(alg, P):
+def test_loopback_driver_matches_oracle(alg, P, gather):
+    """Both exchanges: full-array all-reduce, and the all-gather of owned slices."""
     g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
     s = gg.first_source(g)
-    _, parts = make_parts(g, P)
-    labels, st = edist.run_partitions(parts, edist.LoopbackGroup(), ALGS[alg], s)
+    bounds, parts = make_parts(g, P)
+    labels, st = edist.run_partitions(parts, edist.LoopbackGroup(), ALGS[alg], s,
+                                      bounds if gather else None)
     np.testing.assert_array_equal(labels.numpy().view(np.uint32), expected(alg, g, s))
     if alg == "bfs":
         assert st.edges_processed == int(np.diff(g.off.numpy())[expected(alg, g, s) != oracle.INF].sum())
 
 
-def _gloo_worker(rank, world, port, alg, out):
+def _gloo_worker(rank, world, port, alg, out, gather=False):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -82,16 +85,17 @@ def _gloo_worker(rank, world, port, alg, out):
     bounds = edist.partition_ranges(g.off, g.col, g.n, world)
     loff, lcol, lw = edist.partition_csr(g.off, g.col, g.w, g.n, bounds[rank], bounds[rank + 1])
     eng = MockEngine(loff.numpy(), lcol.numpy(), None if lw is None else lw.numpy(), g.n)
-    labels, st = edist.run_partitions([eng], edist.TorchDistGroup(), ALGS[alg], s)
+    labels, st = edist.run_partitions([eng], edist.TorchDistGroup(), ALGS[alg], s, bounds if gather else None)
     torch.save(labels, out + f".{rank}")
     dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("gather", [False, True])
 @pytest.mark.parametrize("alg", ["bfs", "sssp", "cc"])
-def test_gloo_world2_matches_oracle(alg, tmp_path):
-    port = 29500 + (os.getpid() % 1000) + ALGS[alg]
+def test_gloo_world2_matches_oracle(alg, gather, tmp_path):
+    port = 29500 + (os.getpid() % 1000) + ALGS[alg] + (8 if gather else 0)
     out = str(tmp_path / "labels")
-    mp.spawn(_gloo_worker, args=(2, port, alg, out), nprocs=2, join=True)
+    mp.spawn(_gloo_worker, args=(2, port, alg, out, gather), nprocs=2, join=True)
     g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
     exp = expected(alg, g, gg.first_source(g))
     for r in range(2):

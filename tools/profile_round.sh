@@ -12,3 +12,7 @@ ncu --set full --clock-control none --import-source on -k regex:expand_warp -s 3
 ncu --set full --clock-control none --import-source on -k regex:expand_warp -s 4 -c 1 -o gpurun_out/ncu_expand_sssp_$tag \
     python tools/prof_run.py --algs sssp > gpurun_out/ncu_expand_sssp_$tag.log 2>&1
 ls -la gpurun_out/*$tag*
+# warm-cache launch list (no cache flush between kernels: closer to the graph run)
+ncu --metrics gpu__time_duration.sum --clock-control none --cache-control none -k regex:"expand|udc_scan|init_kernel|ctl_begin" --csv \
+    --log-file gpurun_out/launches_warm_$tag.csv python tools/prof_run.py --algs bfs,sssp,cc > /dev/null 2>&1
+python tools/iter_trace.py --algs bfs,sssp,cc --json gpurun_out/trace_$tag.json > gpurun_out/trace_$tag.log 2>&1
