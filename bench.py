@@ -520,8 +520,8 @@ def run_ours(args):
 
 def run_partitioned(args):
     """One graph split over the N ranks: every rank expands the
-    replicated active set over its destination partition; NCCL all-reduce
-    exchange per iteration.  Strong scaling: the same traversals at every N."""
+    replicated active set over its destination partition; NCCL all-gather of
+    the owned bitmap words / labels per iteration.  Strong scaling: the same traversals at every N."""
     import torch
     import torch.distributed as tdist
     import graphgen as gg
@@ -583,7 +583,7 @@ def run_partitioned(args):
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
             "config": {"workload": config_desc(args.config) + "; " + "+".join(algs) + " per step",
-                       "parallelism": f"1-D destination partition over {world} GPU(s), NCCL all-reduce exchange",
+                       "parallelism": f"1-D destination partition over {world} GPU(s), NCCL all-gather exchange of owned slices",
                        "K": args.K, "flags": args.flags},
             "per_alg": {k: {"gteps": v["gteps"], "ms_per_call": v["ms_per_call"]} for k, v in res.items()},
         }
