@@ -185,6 +185,11 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.prefetch = g->p.prefetch ? 1u : 0u;
     d.ahead = g->p.ahead ? 1u : 0u;
     d.K = g->p.K;
+    d.K_log2 = 32;
+    if (d.K && !(d.K & (d.K - 1))) {
+        d.K_log2 = 0;
+        while ((1u << d.K_log2) < d.K) ++d.K_log2;
+    }
     d.ts = g->p.ts;
     d.ts_log2 = g->p.ts_log2;
     d.tune = g->tune;

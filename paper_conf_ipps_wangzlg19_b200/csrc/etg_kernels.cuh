@@ -106,6 +106,7 @@ struct Dev {
     uint32_t n;
     uint32_t nwords;            // bitmap words (padded to whole scan tiles)
     uint32_t K;                 // degree limit (Def. 3); unused with NO_UDC
+    uint32_t K_log2;            // log2(K) when K is a power of two, else 32
     uint32_t ts;                // shadows per expand tile (<= kBlock, power of 2)
     uint32_t ts_log2;
     uint32_t tune;              // experiment switches (ETG_TUNE env var at load); 0 = default
@@ -244,10 +245,15 @@ __device__ __forceinline__ T block_excl_scan(T x, T *wsum, T &total) {
 
 // Number of shadow vertices of a vertex of out-degree `deg` (Def. 3; L142:
 // degree 0 gives none).
+// ceil(deg / K) as a shift when K is a power of two (klog < 32): the scan
+// evaluates it twice per active vertex, and a runtime integer division is a
+// ~20-instruction sequence.
 template <bool UDC, class D>
-__device__ __forceinline__ uint32_t udc_count(D deg, uint32_t K) {
-    if (UDC) return (uint32_t)((deg + (D)K - 1) / (D)K);
-    return deg > 0 ? 1u : 0u;
+__device__ __forceinline__ uint32_t udc_count(D deg, uint32_t K, uint32_t klog) {
+    if (!UDC) return deg > 0 ? 1u : 0u;
+    if (deg == 0) return 0u;
+    if (klog < 32) return (uint32_t)(((deg - 1) >> klog) + 1);
+    return (uint32_t)((deg - 1) / (D)K + 1);
 }
 
 // ------------------------------------------------------------------------- //
@@ -516,7 +522,7 @@ __global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGr
                 for (int r = 0; r < kG; ++r) {
                     if (!word[r]) continue;
                     nbits += __popc(word[r]);
-                    const uint32_t c = ((word[r] >> lane) & 1u) ? udc_count<UDC>((uint32_t)(oe[r] - ob[r]), d.K) : 0u;
+                    const uint32_t c = ((word[r] >> lane) & 1u) ? udc_count<UDC>((uint32_t)(oe[r] - ob[r]), d.K, d.K_log2) : 0u;
                     const uint32_t kept = __ballot_sync(kFull, c > 0);
                     wsum += ((u64)__popc(kept) << 32) | __reduce_add_sync(kFull, c);
                 }
@@ -610,7 +616,7 @@ __global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGr
                         else if (label && qmark) d.snap[v] = lv[r];   // refresh the snapshot (Q-mark mode)
                     }
                     const uint32_t dg = (uint32_t)(oe[r] - ob[r]);
-                    const uint32_t c = bit ? udc_count<UDC>(dg, d.K) : 0u;
+                    const uint32_t c = bit ? udc_count<UDC>(dg, d.K, d.K_log2) : 0u;
                     const uint32_t kept = __ballot_sync(kFull, c > 0);
                     const uint32_t cincl = warp_incl_scan(c);
                     if (c) {
