@@ -58,6 +58,7 @@ struct Params {
     bool prefetch;  // warp kernel: L2 bulk prefetch of the next tile's segments (ETG_TUNE 128)
     bool ahead;     // warp kernel: next batch's segments loaded one batch ahead (SMP; off: ETG_NO_SMP)
     bool u64;
+    bool persist;   // the iteration loop as one persistent cooperative kernel (loop_kernel)
     uint32_t nf_delta;  // near-far SSSP bucket width (0 = paper schedule)
 };
 
@@ -93,6 +94,7 @@ Params derive(const etg_options *opt, uint32_t tune) {
         // look-ahead alone, so it is an experiment switch only
         p.prefetch = p.udc && (tune & 128u) && !(flags & ETG_NO_SMP) && !p.smp && !host_edges;
     }
+    p.persist = p.warp && !p.smp && (tune & kTunePersist);
     p.ts_log2 = 0;
     while ((1u << p.ts_log2) < p.ts) ++p.ts_log2;
     return p;
@@ -156,6 +158,7 @@ struct etg_graph {
     uint64_t step_launches = 0;
     uint64_t step_acts = 0;               // activations counted so far (cumulative)
     cudaGraphExec_t exec[4] = {nullptr, nullptr, nullptr, nullptr};
+    int grid_loop[4] = {0, 0, 0, 0};      // loop_kernel grid per algorithm (resident CTAs x SMs)
     cudaGraph_t graph[4] = {nullptr, nullptr, nullptr, nullptr};
 };
 
@@ -193,6 +196,17 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.ts = g->p.ts;
     d.ts_log2 = g->p.ts_log2;
     d.tune = g->tune;
+    d.snap_used = 0;
+    return d;
+}
+
+// Dev of the fused single-GPU loop: the snapshot also records the label each
+// sole shadow expanded with (not in the step-wise path, whose ranks must
+// agree on the activated set).
+template <class OffT>
+Dev<OffT> make_dev_fused(const etg_graph *g, int alg) {
+    Dev<OffT> d = make_dev<OffT>(g, alg);
+    d.snap_used = (alg != ALG_BFS && !(g->tune & (kTuneQMark | kTuneNoSnapUsed))) ? 1u : 0u;
     return d;
 }
 
@@ -227,6 +241,21 @@ const void *expand_fn_alg(int alg, bool udc, bool idx, bool smp, bool warp) {
         case ALG_SSSP: return expand_fn<OffT, ALG_SSSP>(udc, idx, smp);
         case ALG_CC: return expand_fn<OffT, ALG_CC>(udc, idx, smp);
         default: return expand_fn<OffT, ALG_SSWP>(udc, idx, smp);
+    }
+}
+
+template <class OffT, int ALG>
+const void *loop_fn_udc(bool udc) {
+    return udc ? (const void *)loop_kernel<OffT, ALG, true> : (const void *)loop_kernel<OffT, ALG, false>;
+}
+
+template <class OffT>
+const void *loop_fn(int alg, bool udc) {
+    switch (alg) {
+        case ALG_BFS: return loop_fn_udc<OffT, ALG_BFS>(udc);
+        case ALG_SSSP: return loop_fn_udc<OffT, ALG_SSSP>(udc);
+        case ALG_CC: return loop_fn_udc<OffT, ALG_CC>(udc);
+        default: return loop_fn_udc<OffT, ALG_SSWP>(udc);
     }
 }
 
@@ -285,7 +314,7 @@ etg_status expand_launch(etg_graph *g, int alg, Launch &out) {
 template <class OffT>
 etg_status build_graph(etg_graph *g, int alg) {
     if (g->exec[alg]) return ETG_OK;
-    Dev<OffT> d = make_dev<OffT>(g, alg);
+    Dev<OffT> d = make_dev_fused<OffT>(g, alg);
     Launch ex;
     etg_status s = expand_launch<OffT>(g, alg, ex);
     if (s != ETG_OK) return s;
@@ -330,13 +359,22 @@ etg_status build_graph(etg_graph *g, int alg) {
 
 template <class OffT>
 etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stats *st) {
-    Dev<OffT> d = make_dev<OffT>(g, alg);
+    Dev<OffT> d = make_dev_fused<OffT>(g, alg);
     cudaStream_t s = g->stream;
     const bool profile = (g->flags & ETG_PROFILE) != 0;
     const bool host_loop = profile || (g->flags & ETG_HOST_LOOP) != 0;
     float scan_ms = 0.f, expand_ms = 0.f;
     uint32_t expand_launches = 0;
-    if (!host_loop) {
+    const bool persist = !host_loop && g->p.persist;
+    if (persist && !g->grid_loop[alg]) {
+        const void *fn = loop_fn<OffT>(alg, g->p.udc);
+        ETG_CU(cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 0));
+        int nb = 0;
+        ETG_CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, kBlock, 0));
+        if (nb < 1) return fail(ETG_ECUDA, "loop_kernel: no resident CTA");
+        g->grid_loop[alg] = nb * g->num_sms;
+    }
+    if (!host_loop && !persist) {
         etg_status rc = build_graph<OffT>(g, alg);
         if (rc != ETG_OK) return rc;
     }
@@ -353,7 +391,14 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
     // A2 of the initial active set (Proc. 1 "Init actSet")
     ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
     uint64_t launches = 3;
-    if (host_loop) {
+    if (persist) {
+        // the whole loop in one cooperative launch (all CTAs co-resident)
+        const void *fn = loop_fn<OffT>(alg, g->p.udc);
+        uint32_t cap_e = expand_arg(g->p);
+        void *largs[] = {&d, &cap_e};
+        ETG_CU(cudaLaunchCooperativeKernel(fn, dim3((unsigned)g->grid_loop[alg]), dim3(kBlock), largs, 0, s));
+        launches += 1;
+    } else if (host_loop) {
         Launch ex;
         etg_status rc = expand_launch<OffT>(g, alg, ex);
         if (rc != ETG_OK) return rc;
@@ -387,7 +432,7 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
     ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     ETG_CU(cudaStreamSynchronize(s));
     ETG_CU(cudaGetLastError());
-    if (!host_loop) launches += 2ull * g->h_ctl->depth;   // body runs = scans after the first
+    if (!host_loop && !persist) launches += 2ull * g->h_ctl->depth;   // body runs = scans after the first
     g_launches += launches;
     if (st) {
         float ms = 0.f;
@@ -396,6 +441,12 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
         st->expand_launches = expand_launches;
         st->activations = g->h_ctl->activations;
         st->frontier_total = g->h_ctl->frontier;
+        if (persist) {
+            // phase times of the persistent loop (%globaltimer, barrier to barrier)
+            scan_ms = (float)(g->h_ctl->t_scan_ns * 1e-6);
+            expand_ms = (float)(g->h_ctl->t_expand_ns * 1e-6);
+            expand_launches = g->h_ctl->depth;
+        }
         st->scan_ms = scan_ms;
         st->expand_ms = expand_ms;
         st->reserved = 0.f;

@@ -51,6 +51,9 @@ constexpr uint32_t kFull = 0xFFFFFFFFu;
 #ifndef ETG_SGRAB
 #define ETG_SGRAB 1                         // expand: first tile grab static (global warp index)
 #endif
+#ifndef ETG_BAR_SLEEP
+#define ETG_BAR_SLEEP 0                     // persistent loop: ns of back-off per grid-barrier poll
+#endif
 #ifndef ETG_PIPE
 #define ETG_PIPE 1                          // software-pipelined batch loop in the warp expand
 #endif
@@ -84,6 +87,9 @@ struct Ctl {
     uint32_t far_min;     //   min label of the deferred (far) marked vertices of the last scan
     uint32_t far_count;   //   number of deferred marked vertices of the last scan
     uint32_t more;        // loop condition computed by the last scan
+    uint32_t bar;         // persistent loop: grid-barrier arrivals in the current call
+    unsigned long long t_expand_ns;   // persistent loop: %globaltimer time of the expand phases
+    unsigned long long t_scan_ns;     //   ... and of the scan phases (block 0's view, barrier to barrier)
 };
 
 template <class OffT>
@@ -113,6 +119,7 @@ struct Dev {
     uint32_t prefetch;          // warp kernel, direct mode: L2 bulk prefetch of the next tile
     uint32_t ahead;             // warp kernel: stage A of the next batch before stage B of this one
     uint32_t nf_delta;          // near-far SSSP bucket width (0: the paper's schedule)
+    uint32_t snap_used;         // SSSP/CC/SSWP, single GPU: a sole shadow stores the label it expands with
 };
 
 constexpr uint32_t kTuneFilterL1 = 1u;    // pre-filter label loads cached in L1
@@ -121,6 +128,8 @@ constexpr uint32_t kTuneNoGather = 16u;   // skip the label gather and the commi
 constexpr uint32_t kTuneNoCommit = 32u;   // gather labels but never commit (counts passes)
 constexpr uint32_t kTuneQMark = 64u;      // A/B: SSSP/CC/SSWP commits also set Q, the scan reads only Q
 constexpr uint32_t kTuneScanDyn = 256u;   // A/B: every scan tile from the counter (no static first tile)
+constexpr uint32_t kTuneNoSnapUsed = 512u; // A/B: snapshot = labels at the iteration start only
+constexpr uint32_t kTunePersist = 1024u;   // experiment: the loop as one persistent kernel (loop_kernel)
 
 // ------------------------------------------------------------------------- //
 // small device helpers
@@ -128,6 +137,21 @@ constexpr uint32_t kTuneScanDyn = 256u;   // A/B: every scan tile from the count
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
 
 __device__ __forceinline__ uint32_t ld_cg(const uint32_t *p) { return __ldcg(p); }
+
+// Control-block / cross-phase reads.  Separate kernels see each other's
+// writes through L2 (L1 starts cold at every launch); inside the persistent
+// loop kernel (P) a value written by another SM in an earlier phase must not
+// come from a stale L1 line, so those reads bypass L1.
+template <bool P, class T>
+__device__ __forceinline__ T cld(const T &x) {
+    if (P) return *(const volatile T *)&x;
+    return x;
+}
+template <bool P, class T>
+__device__ __forceinline__ T xld(const T *p) {
+    if (P) return __ldcg(p);
+    return *p;
+}
 
 // L1-cached label load (experiment switch kTuneFilterL1).  Labels move
 // monotonically, so a stale copy can only let the filter pass an edge.
@@ -277,6 +301,9 @@ __global__ void ctl_begin_kernel(Ctl *ctl, uint32_t *label, uint32_t source) {
     ctl->thresh = 0xFFFFFFFFu;
     ctl->far_min = 0xFFFFFFFFu;
     ctl->far_count = 0;
+    ctl->bar = 0;
+    ctl->t_expand_ns = 0;
+    ctl->t_scan_ns = 0;
 }
 
 // near-far SSSP: the first threshold (the source has distance 0)
@@ -308,7 +335,7 @@ __global__ __launch_bounds__(kBlock) void init_kernel(Dev<OffT> d, uint32_t *lab
     }
     if (ALG == ALG_BFS) {
         for (uint32_t k = blockIdx.x * kBlock + threadIdx.x; k < d.nwords; k += stride)
-            d.V[k] = (k == (source >> 5)) ? (1u << (source & 31)) : 0u;
+            d.V[k] = 0u;                                  // the first scan moves the source from Q to V
     }
     if (ALG == ALG_CC) {
         for (uint32_t k = blockIdx.x * kBlock + threadIdx.x; k < d.nwords; k += stride) {
@@ -385,9 +412,8 @@ __device__ __forceinline__ void lookback_resolve(const unsigned long long (&r)[N
     else p -= 32 * N;
 }
 
-template <class OffT, bool UDC, bool BFSLAB>
-__global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGraphConditionalHandle cond,
-                                                          int use_cond) {
+template <class OffT, bool UDC, bool BFSLAB, bool P>
+__device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditionalHandle cond, int use_cond) {
     typedef unsigned long long u64;
     __shared__ uint32_t s_tile;
     __shared__ u64 s_prefix;
@@ -395,14 +421,14 @@ __global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGr
     __shared__ uint32_t s_acts;                           // activations of this CTA (one global atomic)
     Ctl *ctl = d.ctl;
     if (threadIdx.x == 0) s_acts = 0;
-    const uint32_t epoch = ctl->epoch & 0x3FFFFFFFu;
+    const uint32_t epoch = cld<P>(ctl->epoch) & 0x3FFFFFFFu;
     const uint32_t nscan = (d.n + kScanV - 1) / kScanV;
     const uint32_t ts = d.ts, tsl = d.ts_log2;
     const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
     const uint32_t lt = (1u << lane) - 1u;
-    uint32_t *label = ctl->label;
-    const uint32_t new_depth = ctl->depth + 1;            // BFS depth of the vertices in Q
-    const uint32_t th = ctl->thresh;                      // near-far threshold (SSSP option)
+    uint32_t *label = cld<P>(ctl->label);
+    const uint32_t new_depth = cld<P>(ctl->depth) + 1;    // BFS depth of the vertices in Q
+    const uint32_t th = cld<P>(ctl->thresh);              // near-far threshold (SSSP option)
     const bool qmark = !d.nf_delta && (d.tune & kTuneQMark);   // A/B switch: the expand marks Q itself
     const bool stat = !(d.tune & kTuneScanDyn);
     for (uint32_t round = 0;; ++round) {
@@ -422,75 +448,68 @@ __global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGr
         // -- near-far SSSP keeps the deferred far bits)
         uint32_t wq[kWPW / 32];
 #pragma unroll
-        for (int j = 0; j < kWPW / 32; ++j) wq[j] = d.Q[wbase + 32 * j + lane];
+        for (int j = 0; j < kWPW / 32; ++j) wq[j] = xld<P>(&d.Q[wbase + 32 * j + lane]);
         uint32_t far_cnt = 0, far_min = kInf;
-        if (d.nf_delta) {
-            // near-far: marked vertices with label >= thresh stay marked (deferred)
+        const bool nf = d.nf_delta != 0;
+#pragma unroll
+        for (int j = 0; j < kWPW / 32; ++j)
+            if (wq[j]) {
+                d.Q[wbase + 32 * j + lane] = 0u;
+                if (BFSLAB) {
+                    // visited from now on (depth written below).  Only bits not
+                    // yet in V are new: an expand that read a stale V line (the
+                    // persistent loop) may have marked a visited vertex again.
+                    const uint32_t vw = xld<P>(&d.V[wbase + 32 * j + lane]);
+                    wq[j] &= ~vw;
+                    if (wq[j]) d.V[wbase + 32 * j + lane] = vw | wq[j];
+                }
+            }
+        if (!BFSLAB && label && !qmark) {
+            // SSSP/CC/SSWP: a vertex is active iff its label moved since it
+            // was last expanded (label != snap; the expand marks nothing for
+            // them), or init/exchange put it in Q.  Word k of the warp = the
+            // ballot over vertices 32k .. 32k+31: coalesced label/snap loads.
+            // Near-far SSSP: a moved vertex at distance >= thresh is deferred
+            // -- its snapshot is not refreshed, so it stays "moved" and is
+            // looked at again by every later scan until the threshold passes it.
 #pragma unroll
             for (int j = 0; j < kWPW / 32; ++j) {
-                uint32_t keep_far = 0;
-                for (uint32_t k = 0; k < 32; ++k) {
-                    const uint32_t word = __shfl_sync(kFull, wq[j], k);
-                    if (!word) continue;
-                    const bool bit = (word >> lane) & 1u;
-                    const uint32_t v = (wbase + 32 * j + k) * 32 + lane;
-                    uint32_t lv = 0;
-                    if (bit) {
-                        lv = __ldcg(&label[v]);
-                        d.snap[v] = lv;                   // refresh the pre-filter snapshot
-                    }
-                    const uint32_t far = __ballot_sync(kFull, bit && lv >= th);
-                    if (far) {
-                        if (bit && lv >= th) far_min = min(far_min, lv);
-                        if (lane == k) keep_far = far;
-                    }
-                    far_cnt += __popc(far);
-                }
-                if (wq[j] | keep_far) d.Q[wbase + 32 * j + lane] = keep_far;
-                wq[j] &= ~keep_far;
-            }
-            far_min = __reduce_min_sync(kFull, far_min);
-            if (lane == 0 && far_cnt) {
-                atomicAdd(&ctl->far_count, far_cnt);
-                atomicMin(&ctl->far_min, far_min);
-            }
-            __threadfence();                              // before this tile publishes
-        } else {
+                uint32_t mine = 0;
+                for (uint32_t k0 = 0; k0 < 32; k0 += 2 * kG) {
+                    uint32_t lv[2 * kG], sv[2 * kG];
 #pragma unroll
-            for (int j = 0; j < kWPW / 32; ++j)
-                if (wq[j]) {
-                    d.Q[wbase + 32 * j + lane] = 0u;
-                    if (BFSLAB) d.V[wbase + 32 * j + lane] |= wq[j];   // visited from now on (depth written below)
-                }
-            if (!BFSLAB && label && !(d.tune & kTuneQMark)) {
-                // SSSP/CC/SSWP: a vertex is active iff its label moved since it
-                // was last expanded (label != snap; the expand marks nothing for
-                // them), or init/exchange put it in Q.  Word k of the warp = the
-                // ballot over vertices 32k .. 32k+31: coalesced label/snap loads.
-#pragma unroll
-                for (int j = 0; j < kWPW / 32; ++j) {
-                    uint32_t mine = 0;
-                    for (uint32_t k0 = 0; k0 < 32; k0 += 2 * kG) {
-                        uint32_t lv[2 * kG], sv[2 * kG];
-#pragma unroll
-                        for (int r = 0; r < 2 * kG; ++r) {
-                            const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
-                            lv[r] = 0;
-                            sv[r] = 0;
-                            if (v < d.n) {
-                                lv[r] = __ldcg(&label[v]);
-                                sv[r] = __ldcg(&d.snap[v]);
-                            }
-                        }
-#pragma unroll
-                        for (int r = 0; r < 2 * kG; ++r) {
-                            const uint32_t b = __ballot_sync(kFull, lv[r] != sv[r]);
-                            if (lane == k0 + r) mine = b;
-                            if (lv[r] != sv[r]) d.snap[(wbase + 32 * j + k0 + r) * 32 + lane] = lv[r];   // refresh
+                    for (int r = 0; r < 2 * kG; ++r) {
+                        const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
+                        lv[r] = 0;
+                        sv[r] = 0;
+                        if (v < d.n) {
+                            lv[r] = __ldcg(&label[v]);
+                            sv[r] = __ldcg(&d.snap[v]);
                         }
                     }
-                    wq[j] |= mine;
+#pragma unroll
+                    for (int r = 0; r < 2 * kG; ++r) {
+                        const bool moved = lv[r] != sv[r];
+                        const bool far = nf && moved && lv[r] >= th;
+                        const uint32_t b = __ballot_sync(kFull, moved && !far);
+                        if (lane == k0 + r) mine = b;
+                        if (moved && !far) d.snap[(wbase + 32 * j + k0 + r) * 32 + lane] = lv[r];   // refresh
+                        if (far) {
+                            ++far_cnt;
+                            far_min = min(far_min, lv[r]);
+                        }
+                    }
                 }
+                wq[j] |= mine;
+            }
+            if (nf) {
+                far_cnt = __reduce_add_sync(kFull, far_cnt);
+                far_min = __reduce_min_sync(kFull, far_min);
+                if (lane == 0 && far_cnt) {
+                    atomicAdd(&ctl->far_count, far_cnt);
+                    atomicMin(&ctl->far_min, far_min);
+                }
+                __threadfence();                          // before this tile publishes
             }
         }
         // pass 1: this warp's (kept, shadows); groups of kG words, all offset
@@ -642,12 +661,12 @@ __global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGr
             ctl->nshadow = N;
             ctl->ntiles = (N + ts - 1) >> tsl;
             ctl->tile_ctr = 0;
-            ctl->depth += 1;
+            ctl->depth = cld<P>(ctl->depth) + 1;
             bool more = nF > 0;
-            if (d.nf_delta && ctl->far_count) {
+            if (d.nf_delta && cld<P>(ctl->far_count)) {
                 more = true;
                 if (nF == 0) {                        // near set empty: next bucket
-                    const unsigned long long thn = (unsigned long long)ctl->far_min + d.nf_delta;
+                    const unsigned long long thn = (unsigned long long)cld<P>(ctl->far_min) + d.nf_delta;
                     ctl->thresh = thn > kInf ? kInf : (uint32_t)thn;
                 }
             }
@@ -658,6 +677,12 @@ __global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGr
         __syncthreads();
     }
     if (threadIdx.x == 0 && s_acts) atomicAdd(&ctl->activations, (u64)s_acts);   // result unused: RED
+}
+
+template <class OffT, bool UDC, bool BFSLAB>
+__global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGraphConditionalHandle cond,
+                                                          int use_cond) {
+    scan_phase<OffT, UDC, BFSLAB, false>(d, cond, use_cond);
 }
 
 // ------------------------------------------------------------------------- //
@@ -868,7 +893,7 @@ __global__ __launch_bounds__(kBlock) void expand_kernel(Dev<OffT> d, uint32_t ca
                 cur[r] = act[r] ? (l1 ? ld_ca(&label[u[r]]) : ld_cg(&label[u[r]])) : 0u;
 #pragma unroll
             for (int r = 0; r < kR; ++r)
-                if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, d.nf_delta != 0 || (d.tune & kTuneQMark));
+                if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, (d.tune & kTuneQMark) != 0);
         }
         my_edges += E;
         __syncthreads();
@@ -893,21 +918,22 @@ struct WarpShadow {
     OffT start;
     uint32_t len;
     uint32_t v;
+    bool sole;         // the vertex's only shadow (its whole row)
 };
 
-template <class OffT, bool UDC>
+template <class OffT, bool UDC, bool P = false>
 __device__ __forceinline__ WarpShadow<OffT, UDC> warp_map(const Dev<OffT> &d, uint32_t t, uint32_t nF,
                                                           uint32_t N) {
     const uint32_t lane = lane_id();
-    const uint32_t j0 = d.tile_first[t];
+    const uint32_t j0 = xld<P>(&d.tile_first[t]);
     const uint32_t j = j0 + lane;
     uint32_t Sj = kInf, Dj = 0, Fj = 0;
     OffT Bj = 0;
     if (j < nF) {
-        Sj = d.S[j];
-        Bj = d.B[j];
-        Dj = d.D[j];
-        Fj = d.F[j];
+        Sj = xld<P>(&d.S[j]);
+        Bj = xld<P>(&d.B[j]);
+        Dj = xld<P>(&d.D[j]);
+        Fj = xld<P>(&d.F[j]);
     }
     const uint32_t base = t << 5;
     const uint32_t p = Sj - base;                              // wraps to huge if Sj < base
@@ -920,6 +946,7 @@ __device__ __forceinline__ WarpShadow<OffT, UDC> warp_map(const Dev<OffT> &d, ui
     r.v = __shfl_sync(kFull, Fj, jj);
     r.len = 0;
     r.start = 0;
+    r.sole = !UDC || sD <= d.K;
     const uint32_t i = base + lane;
     if (i < N) {
         if (UDC) {
@@ -972,16 +999,16 @@ struct WarpTile {
     uint32_t sdelta;   // ... and stage[sdelta + x] in shared memory            (SMP)
 };
 
-template <class OffT, int ALG, bool UDC, bool SMP>
-__global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT> d, uint32_t capw) {
+template <class OffT, int ALG, bool UDC, bool SMP, bool P>
+__device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) {
     constexpr bool kW = (ALG == ALG_SSSP || ALG == ALG_SSWP);
     constexpr uint32_t kArrays = kW ? 2u : 1u;
     constexpr int kRB = kW ? ETG_KR_W : kR;                // chunks per batch (weighted: fewer, no spills)
     extern __shared__ __align__(128) uint8_t dyn_smem[];
     Ctl *ctl = d.ctl;
-    const uint32_t nF = ctl->nF, N = ctl->nshadow, ntiles = ctl->ntiles;
-    const uint32_t level = ctl->depth + 1;
-    uint32_t *label = ctl->label;
+    const uint32_t nF = cld<P>(ctl->nF), N = cld<P>(ctl->nshadow), ntiles = cld<P>(ctl->ntiles);
+    const uint32_t level = cld<P>(ctl->depth) + 1;
+    uint32_t *label = cld<P>(ctl->label);
     uint32_t *Q = d.Q;
     const uint32_t lane = lane_id();
     const uint32_t lt_eq = (2u << lane) - 1u;
@@ -992,12 +1019,12 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         // bookkeeping for the scan that follows this kernel (stream-ordered)
         ctl->scan_ctr = 0;
-        ctl->epoch += 1;
+        ctl->epoch = cld<P>(ctl->epoch) + 1;
         ctl->far_min = kInf;
         ctl->far_count = 0;
-        if (nF) ctl->iterations += 1;
-        ctl->frontier += nF;
-        ctl->shadows += N;
+        if (nF) ctl->iterations = cld<P>(ctl->iterations) + 1;
+        ctl->frontier = cld<P>(ctl->frontier) + nF;
+        ctl->shadows = cld<P>(ctl->shadows) + N;
     }
     // SMP: two shared-memory stages per warp, each kArrays x capw words, and
     // one mbarrier per stage (the TMA bulk copies complete on it).
@@ -1046,7 +1073,7 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
     // shared memory before processing them); direct -> L2 bulk prefetch.
     auto prepare = [&](uint32_t t, uint32_t st) -> WarpTile<OffT, UDC> {
         WarpTile<OffT, UDC> w;
-        w.sh = warp_map<OffT, UDC>(d, t, nF, N);
+        w.sh = warp_map<OffT, UDC, P>(d, t, nF, N);
         const uint32_t incl = warp_incl_scan(w.sh.len);
         w.o = incl - w.sh.len;
         w.E = __shfl_sync(kFull, incl, 31);
@@ -1103,7 +1130,7 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
     // flight while the gathers of this one are: one memory latency per batch
     // instead of two.  Stage B needs only registers, so a tile's shared-memory
     // stage (SMP) can be refilled once stage A has left the tile.
-    const bool markQ = d.nf_delta != 0 || (d.tune & kTuneQMark);
+    const bool markQ = (d.tune & kTuneQMark) != 0;   // near-far defers through the snapshot, not Q
     const uint32_t *filt = (ALG == ALG_BFS) ? label : d.snap;   // BFS: live labels; else snapshot (R-4, R-6)
     uint32_t t = next_tile();
     if (t < ntiles) {
@@ -1113,7 +1140,17 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
         uint32_t kt = 0;
         uint32_t tn = next_tile();
         if (tn < ntiles) nxt = prepare(tn, 1);
-        uint32_t A_lab = (ALG == ALG_BFS) ? level : (A_t.sh.len ? ld_cg(&label[A_t.sh.v]) : 0u);
+        // fresh source label (R-6).  Single GPU: a vertex expanded by a sole
+        // shadow records the label it propagates in the snapshot, so the scan
+        // re-activates it only if its label moves after this read (R-5).
+        const bool snap_used = ALG != ALG_BFS && d.snap_used;
+        auto src_label = [&](const WarpShadow<OffT, UDC> &sh) -> uint32_t {
+            if (!sh.len) return 0u;
+            const uint32_t l = ld_cg(&label[sh.v]);
+            if (snap_used && sh.sole) d.snap[sh.v] = l;
+            return l;
+        };
+        uint32_t A_lab = (ALG == ALG_BFS) ? level : src_label(A_t.sh);
         uint32_t A_x0 = 0, A_owner = 0xFFFFFFFFu;
         const uint32_t *A_sbuf = nullptr;
         if (SMP) {
@@ -1176,7 +1213,7 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
                     ++kt;
                     tn = next_tile();
                     if (tn < ntiles) nxt = prepare(tn, (kt + 1) & 1);   // refills the stage of tile kt-1
-                    A_lab = (ALG == ALG_BFS) ? level : (A_t.sh.len ? ld_cg(&label[A_t.sh.v]) : 0u);
+                    A_lab = (ALG == ALG_BFS) ? level : src_label(A_t.sh);
                     A_x0 = 0;
                     A_owner = 0xFFFFFFFFu;
                     my_edges += A_t.E;
@@ -1203,7 +1240,7 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
                 // kernel, cached in L1: hits never reach the L2 request path)
 #pragma unroll
                 for (int r = 0; r < kRB; ++r)
-                    cur[r] = ((am >> r) & 1u) ? (((__ldg(&d.V[u[r] >> 5]) >> (u[r] & 31)) & 1u) ? 0u : kInf) : 0u;
+                    cur[r] = ((am >> r) & 1u) ? ((((P ? ld_ca(&d.V[u[r] >> 5]) : __ldg(&d.V[u[r] >> 5])) >> (u[r] & 31)) & 1u) ? 0u : kInf) : 0u;
             } else if (ALG == ALG_CC && level == 1) {
                 // CC's first expand: the snapshot is still the initial labelling
                 // label[u] = u (A1), so the pre-filter needs no gather at all
@@ -1330,7 +1367,7 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
                 }
 #pragma unroll
                 for (int r = 0; r < kRB; ++r)
-                    if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, d.nf_delta != 0 || (d.tune & kTuneQMark));
+                    if (act[r] && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, (d.tune & kTuneQMark) != 0);
             }
             if (tn >= ntiles) break;
         }
@@ -1346,6 +1383,69 @@ __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT>
     if (d.tune & kTuneNoCommit) {
         my_passes = __reduce_add_sync(kFull, my_passes);
         if (lane == 0 && my_passes) atomicAdd(&ctl->reached_v, (unsigned long long)my_passes);
+    }
+}
+
+template <class OffT, int ALG, bool UDC, bool SMP>
+__global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT> d, uint32_t capw) {
+    expand_phase<OffT, ALG, UDC, SMP, false>(d, capw);
+}
+
+// ------------------------------------------------------------------------- //
+// A6 as one persistent kernel: the whole "while actSet.isNotEmpty()" loop of
+// Proc. 1 (L207) -- expand (A2-A5), grid barrier, scan (A5 + A2 of the next
+// iteration), grid barrier -- in one cooperative launch, so an iteration pays
+// two barriers instead of two kernel launches.  Same phase code as the
+// separate kernels; cross-phase reads bypass L1 (P = true).
+// ------------------------------------------------------------------------- //
+__device__ __forceinline__ unsigned long long globaltimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
+// Grid barrier over a monotone arrival counter (zeroed by ctl_begin_kernel):
+// barrier k of the call completes when the counter reaches k * gridDim.x.
+// Release on arrival, acquire on exit.  All CTAs are co-resident (cooperative
+// launch), so it cannot deadlock; a spin longer than ~10 s traps instead of
+// hanging the device.
+__device__ __forceinline__ void grid_barrier(uint32_t *bar, uint32_t &k) {
+    __syncthreads();
+    ++k;
+    if (threadIdx.x == 0) {
+        const uint32_t target = k * gridDim.x;
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(bar) : "memory");
+        const long long t0 = clock64();
+        for (;;) {
+            uint32_t v;
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
+            if ((int)(v - target) >= 0) break;
+            if (clock64() - t0 > 20000000000ll) __trap();
+#if ETG_BAR_SLEEP
+            __nanosleep(ETG_BAR_SLEEP);
+#endif
+        }
+    }
+    __syncthreads();
+}
+
+template <class OffT, int ALG, bool UDC>
+__global__ __launch_bounds__(kBlock, ETG_MINB) void loop_kernel(Dev<OffT> d, uint32_t capw) {
+    Ctl *ctl = d.ctl;
+    uint32_t k = 0;
+    const bool timer = blockIdx.x == 0 && threadIdx.x == 0;
+    while (cld<true>(ctl->more)) {
+        const unsigned long long t0 = timer ? globaltimer() : 0ull;
+        expand_phase<OffT, ALG, UDC, false, true>(d, capw);
+        grid_barrier(&ctl->bar, k);
+        const unsigned long long t1 = timer ? globaltimer() : 0ull;
+        scan_phase<OffT, UDC, ALG == ALG_BFS, true>(d, 0, 0);
+        grid_barrier(&ctl->bar, k);
+        if (timer) {
+            const unsigned long long t2 = globaltimer();
+            ctl->t_expand_ns = cld<true>(ctl->t_expand_ns) + (t1 - t0);
+            ctl->t_scan_ns = cld<true>(ctl->t_scan_ns) + (t2 - t1);
+        }
     }
 }
 
