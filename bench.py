@@ -65,6 +65,10 @@ def parse_args():
     p.add_argument("--partitioned", action="store_true",
                    help="1-D destination partition of ONE graph over the N ranks (NCCL exchange); "
                         "default: N independent replicas")
+    p.add_argument("--push", choices=["off", "auto", "sparse", "dense"], default="off",
+                   help="with --partitioned: SSSP/CC on a SOURCE partition with the push exchange (NEXT-3: "
+                        "all-to-all of proposals / dense reduce-scatter; auto picks per iteration); BFS keeps "
+                        "the destination partition")
     return p.parse_args()
 
 
@@ -549,8 +553,14 @@ def run_partitioned(args):
                 else:
                     d0.init_process_group("nccl", init_method="tcp://127.0.0.1:29555", rank=0,
                                           world_size=1, device_id=dev)
-        dg = edist.DistGraph(g.off, g.col, g.w, g.n, rank, world, K=args.K, flags=args.flags,
-                             symmetric=(a == "cc"), device=dev, group=group)
+        push = args.push != "off" and a != "bfs"
+        if push:
+            dg = edist.PushDistGraph(g.off, g.col, g.w, g.n, rank, world, K=args.K, flags=args.flags,
+                                     symmetric=(a == "cc"), device=dev, group=group, mode=args.push)
+        else:
+            dg = edist.DistGraph(g.off, g.col, g.w, g.n, rank, world, K=args.K, flags=args.flags,
+                                 symmetric=(a == "cc"), device=dev, group=group)
+        lo, hi = dg.bounds[rank], dg.bounds[rank + 1]
         m_sym = g.m
         del g
         torch.cuda.empty_cache()
@@ -567,9 +577,15 @@ def run_partitioned(args):
             if i >= args.warmup:
                 ms_tot += ev0.elapsed_time(ev1)
                 unreached = etg.INF
-                reached = labels.view(torch.int32) != -1 if a != "cc" else None
-                edges_tot += m_sym if a == "cc" else int(deg[reached].sum())
+                if a == "cc":
+                    edges_tot += m_sym
+                elif push:      # owned slice only (summed over the ranks below)
+                    edges_tot += int(deg[lo:hi][labels[lo:hi].view(torch.int32) != -1].sum())
+                else:
+                    edges_tot += int(deg[labels.view(torch.int32) != -1].sum())
         ms_max = allreduce([ms_tot], tdist.ReduceOp.MAX, world)[0] if world > 1 else ms_tot
+        if push and a != "cc" and world > 1:
+            edges_tot = int(allreduce([float(edges_tot)], tdist.ReduceOp.SUM, world)[0])
         res[a] = {"gteps": edges_tot / ms_max / 1e6, "ms_per_call": ms_max / args.steps, "edges": edges_tot,
                   "ms": ms_max}
         del dg, deg
@@ -583,7 +599,10 @@ def run_partitioned(args):
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
             "config": {"workload": config_desc(args.config) + "; " + "+".join(algs) + " per step",
-                       "parallelism": f"1-D destination partition over {world} GPU(s), NCCL all-gather exchange of owned slices",
+                       "parallelism": (f"1-D destination partition over {world} GPU(s), NCCL all-gather exchange of owned slices"
+                                       if args.push == "off" else
+                                       f"SSSP/CC: 1-D source partition over {world} GPU(s), push exchange ({args.push}: "
+                                       f"NCCL all-to-all of proposals or reduce-scatter of labels); BFS: destination partition"),
                        "K": args.K, "flags": args.flags},
             "per_alg": {k: {"gteps": v["gteps"], "ms_per_call": v["ms_per_call"]} for k, v in res.items()},
         }

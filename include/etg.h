@@ -179,6 +179,34 @@ etg_status etg_step_expand(etg_graph *g);
 etg_status etg_step_scan(etg_graph *g, uint32_t *n_active);
 etg_status etg_step_end(etg_graph *g, etg_stats *st_or_null);
 etg_status etg_bitmap_layout(etg_graph *g, size_t *offset_bytes, uint32_t *nwords);
+
+/* ---- NEXT-3 push exchange (the all-to-all option of the
+ * north star's item 4).  SOURCE partition: a rank's handle is loaded with the
+ * out-edges of its owned range [bounds[rank], bounds[rank+1]) only (other
+ * rows empty, global ids), so its relaxations (Proc. 1 L207) land on any
+ * vertex.  SSSP/CC/SSWP only (BFS keeps the destination partition), no
+ * near-far.  After etg_step_expand, every vertex v this rank does NOT own whose
+ * label moved (label != snapshot) carries a proposal for v's owner:
+ *   etg_push_count: d_counts[q] = number of proposals for owner q
+ *     (device, P entries of uint64, overwritten; d_counts[rank] = 0).
+ *   etg_push_pack: appends (v, label[v]) uint32 pairs to d_pairs, owner q's
+ *     proposals at pair index d_cursor[q] onwards (device, P uint64 entries,
+ *     typically the exclusive scan of the counts; advanced by the call; order
+ *     inside a segment unspecified), and marks them sent (snapshot = label).
+ *   etg_push_apply: label[v] = min(label[v], val) (SSWP: max) for `count`
+ *     received pairs (device memory, 2 * count uint32).
+ * Then etg_step_scan activates the owned vertices whose label moved.  The
+ * caller moves the pairs (all-to-all) or, when that is more bytes, reduces the
+ * full label arrays (MIN; SSWP MAX) onto each owner's range instead, and
+ * stops when the compacted active sets of all ranks are empty
+ * (etg_debug_counters out[1]).  d_bounds: P + 1 uint32 in device memory,
+ * bounds[0] = 0, bounds[P] = n, inner bounds multiples of 32.  Errors:
+ * ETG_EINVAL on NULL pointers, P > 64, rank >= P, or no SSSP/CC/SSWP step run. */
+etg_status etg_push_count(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *d_bounds,
+                          unsigned long long *d_counts);
+etg_status etg_push_pack(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *d_bounds,
+                         unsigned long long *d_cursor, uint32_t *d_pairs);
+etg_status etg_push_apply(etg_graph *g, const uint32_t *d_pairs, uint64_t count);
 /* Tracing (step-wise runs): the device counters as of the last etg_step_* call
  * that synchronised (begin/scan/end): out[0] depth, [1] compacted active-set
  * size |F| (Proc. 1 actSet, L207), [2] shadow vertices of F (Def. 3),

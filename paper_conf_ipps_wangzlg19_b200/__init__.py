@@ -91,6 +91,9 @@ def lib():
             "etg_step_scan": (st, [p, ctypes.POINTER(u32)]),
             "etg_step_end": (st, [p, p]),
             "etg_bitmap_layout": (st, [p, ctypes.POINTER(sz), ctypes.POINTER(u32)]),
+            "etg_push_count": (st, [p, u32, u32, p, p]),
+            "etg_push_pack": (st, [p, u32, u32, p, p, p]),
+            "etg_push_apply": (st, [p, p, u64]),
             "etg_debug_expand_replay": (st, [p, ctypes.c_int, u32, u32, u32, ctypes.c_int, p, p,
                                              ctypes.POINTER(ctypes.c_float), ctypes.POINTER(u64),
                                              ctypes.POINTER(u32)]),

@@ -10,6 +10,7 @@
 // reads the active-set size back every iteration (the paper's own control flow).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <atomic>
 #include <cstdio>
 #include <cstdlib>
@@ -155,6 +156,7 @@ struct etg_graph {
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     cudaEvent_t pev[3] = {nullptr, nullptr, nullptr};   // ETG_PROFILE: scan / expand brackets
     int step_alg = -1;                    // algorithm of the step-wise (distributed) run
+    uint32_t *step_label = nullptr;       // its label array
     uint64_t step_launches = 0;
     uint64_t step_acts = 0;               // activations counted so far (cumulative)
     cudaGraphExec_t exec[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -479,6 +481,7 @@ etg_status step_begin_impl(etg_graph *g, int alg, uint32_t source, uint32_t *lab
     ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), iargs, 0, s));
     g->step_launches = 2;
     g->step_alg = alg;
+    g->step_label = label;
     g->step_acts = 0;
     if (!skip_scan) return step_scan_impl<OffT>(g, n_active);
     ETG_CU(cudaStreamSynchronize(s));
@@ -799,6 +802,51 @@ etg_status etg_step_end(etg_graph *g, etg_stats *st) {
         st->shadows = g->h_ctl->shadows;
         st->edges_processed = g->h_ctl->edges;
     }
+    return ETG_OK;
+}
+
+etg_status etg_push_count(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *d_bounds,
+                          unsigned long long *d_counts) {
+    if (!g || !d_bounds || !d_counts) return fail(ETG_EINVAL, "NULL argument");
+    if (g->step_alg < 0 || g->step_alg == ALG_BFS) return fail(ETG_EINVAL, "no step-wise SSSP/CC/SSWP run in progress");
+    if (P < 1 || P > kPushMaxP || rank >= P) return fail(ETG_EINVAL, "need 1 <= P <= 64 and rank < P");
+    if (g->n == 0) return ETG_OK;
+    cudaStream_t s = g->stream;
+    ETG_CU(cudaMemsetAsync(d_counts, 0, sizeof(unsigned long long) * P, s));
+    const uint32_t *label = g->step_label;
+    uint32_t *snap = reinterpret_cast<uint32_t *>(g->ws + g->L.snap);
+    push_pack_kernel<false><<<g->grid_init, kBlock, 0, s>>>(label, snap, (uint32_t)g->n, d_bounds, P, rank,
+                                                            d_counts, nullptr);
+    ETG_CU(cudaGetLastError());
+    g->step_launches += 1;
+    return ETG_OK;
+}
+
+etg_status etg_push_pack(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *d_bounds,
+                         unsigned long long *d_cursor, uint32_t *d_pairs) {
+    if (!g || !d_bounds || !d_cursor || !d_pairs) return fail(ETG_EINVAL, "NULL argument");
+    if (g->step_alg < 0 || g->step_alg == ALG_BFS) return fail(ETG_EINVAL, "no step-wise SSSP/CC/SSWP run in progress");
+    if (P < 1 || P > kPushMaxP || rank >= P) return fail(ETG_EINVAL, "need 1 <= P <= 64 and rank < P");
+    if (g->n == 0) return ETG_OK;
+    uint32_t *snap = reinterpret_cast<uint32_t *>(g->ws + g->L.snap);
+    push_pack_kernel<true><<<g->grid_init, kBlock, 0, g->stream>>>(g->step_label, snap, (uint32_t)g->n, d_bounds,
+                                                                   P, rank, d_cursor, d_pairs);
+    ETG_CU(cudaGetLastError());
+    g->step_launches += 1;
+    return ETG_OK;
+}
+
+etg_status etg_push_apply(etg_graph *g, const uint32_t *d_pairs, uint64_t count) {
+    if (!g || (!d_pairs && count)) return fail(ETG_EINVAL, "NULL argument");
+    if (g->step_alg < 0 || g->step_alg == ALG_BFS) return fail(ETG_EINVAL, "no step-wise SSSP/CC/SSWP run in progress");
+    if (!count) return ETG_OK;
+    const unsigned blocks = (unsigned)std::min<uint64_t>((count + kBlock - 1) / kBlock, (uint64_t)g->grid_init);
+    if (g->step_alg == ALG_SSWP)
+        push_apply_kernel<ALG_SSWP><<<blocks, kBlock, 0, g->stream>>>(g->step_label, d_pairs, count);
+    else
+        push_apply_kernel<ALG_SSSP><<<blocks, kBlock, 0, g->stream>>>(g->step_label, d_pairs, count);
+    ETG_CU(cudaGetLastError());
+    g->step_launches += 1;
     return ETG_OK;
 }
 

@@ -47,13 +47,19 @@ SIGN = -(1 << 31)   # xor with this maps uint32 order onto int32 order
 # --------------------------------------------------------------------------- #
 # partitioning (host logic; torch ops on whatever device the CSR lives on)
 # --------------------------------------------------------------------------- #
-def partition_ranges(off: torch.Tensor, col: torch.Tensor, n: int, P: int, align: int = 32) -> List[int]:
+def partition_ranges(off: torch.Tensor, col: torch.Tensor, n: int, P: int, align: int = 32,
+                     by: str = "in") -> List[int]:
     """Boundaries lo_0 = 0 < ... < lo_P = n, multiples of `align` (except n),
-    balancing in-edge counts.  Returns the P + 1 boundaries."""
+    balancing in-edge counts (by="in": destination partition) or out-edge
+    counts (by="out": source partition, the push exchange).  Returns the P + 1
+    boundaries."""
     if P < 1:
         raise ValueError("P >= 1")
-    indeg = torch.bincount(col.to(torch.int64), minlength=n)
-    cum = torch.cumsum(indeg, 0)
+    if by == "out":
+        deg = (off[1:].to(torch.int64) - off[:-1].to(torch.int64))
+    else:
+        deg = torch.bincount(col.to(torch.int64), minlength=n)
+    cum = torch.cumsum(deg, 0)
     m = int(cum[-1]) if n else 0
     bounds = [0]
     for g in range(1, P):
@@ -93,6 +99,20 @@ def partition_csr(off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor
     return loff, lcol, lw
 
 
+def partition_csr_src(off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor], n: int,
+                      lo: int, hi: int):
+    """The rank's SOURCE-partitioned CSR (push exchange, NEXT-3): rows = all n
+    sources, only the rows of [lo, hi) keep their out-edges (global ids)."""
+    off = off.to(torch.int64)
+    a, b = int(off[lo]), int(off[hi])
+    loff = (off.clamp(min=a, max=b) - a)
+    loff[:lo] = 0
+    loff[hi:] = b - a
+    lcol = col[a:b].to(torch.int32)
+    lw = None if w is None else w[a:b].to(torch.int32)
+    return loff, lcol, lw
+
+
 # --------------------------------------------------------------------------- #
 # collectives
 # --------------------------------------------------------------------------- #
@@ -128,6 +148,47 @@ class TorchDistGroup:
                 t[bounds[q]:bounds[q + 1]] = recv[q][:bounds[q + 1] - bounds[q]]
 
 
+    def alltoallv(self, sends: Sequence[torch.Tensor], counts: Sequence[Sequence[int]]) -> List[torch.Tensor]:
+        """sends[0]: this rank's rows (int32 [k, 2]) grouped by destination rank,
+        counts[0][q] rows for rank q.  Returns [rows received, grouped by source]."""
+        assert len(sends) == 1
+        send, cnt = sends[0], list(counts[0])
+        P = len(cnt)
+        c = torch.tensor(cnt, dtype=torch.int64, device=send.device)
+        rc = torch.empty_like(c)
+        self.dist.all_to_all_single(rc, c, group=self.group)
+        rcnt = [int(x) for x in rc.cpu()]
+        recv = torch.empty((sum(rcnt), send.shape[1]), dtype=send.dtype, device=send.device)
+        if P and (sum(rcnt) or sum(cnt)):
+            self.dist.all_to_all_single(recv, send, output_split_sizes=rcnt, input_split_sizes=cnt,
+                                        group=self.group)
+        return [recv]
+
+    def reduce_ranges(self, tensors: Sequence[torch.Tensor], bounds: Sequence[int], op: str) -> None:
+        """Rank r's slice [bounds[r], bounds[r+1]) becomes the element-wise `op`
+        (min/max, int32 order) over all ranks' tensors; other slices are left
+        as they are.  NCCL: one reduce-scatter of padded slices; gloo (no
+        reduce-scatter): an all-reduce of the whole tensor."""
+        assert len(tensors) == 1
+        t = tensors[0]
+        r = self.dist.get_rank(self.group)
+        P = len(bounds) - 1
+        ops = {"min": self.dist.ReduceOp.MIN, "max": self.dist.ReduceOp.MAX}
+        if self.dist.get_backend(self.group) != "nccl":
+            acc = t.clone()
+            self.dist.all_reduce(acc, op=ops[op], group=self.group)
+            t[bounds[r]:bounds[r + 1]] = acc[bounds[r]:bounds[r + 1]]
+            return
+        width = max(bounds[q + 1] - bounds[q] for q in range(P))
+        pad = 0x7FFFFFFF if op == "min" else -(1 << 31)
+        inp = torch.full((P, width), pad, dtype=t.dtype, device=t.device)
+        for q in range(P):
+            inp[q, :bounds[q + 1] - bounds[q]] = t[bounds[q]:bounds[q + 1]]
+        out = torch.empty(width, dtype=t.dtype, device=t.device)
+        self.dist.reduce_scatter_tensor(out, inp.reshape(-1), op=ops[op], group=self.group)
+        t[bounds[r]:bounds[r + 1]] = out[:bounds[r + 1] - bounds[r]]
+
+
 class LoopbackGroup:
     """P 'ranks' in one process (one GPU): all_reduce over a list of tensors."""
 
@@ -148,6 +209,21 @@ class LoopbackGroup:
             for t in tensors:
                 if t is not src:
                     t[bounds[q]:bounds[q + 1]] = src[bounds[q]:bounds[q + 1]]
+
+
+    def alltoallv(self, sends: Sequence[torch.Tensor], counts: Sequence[Sequence[int]]) -> List[torch.Tensor]:
+        P = len(sends)
+        starts = [[sum(counts[q][:r]) for r in range(P)] for q in range(P)]
+        return [torch.cat([sends[q][starts[q][r]:starts[q][r] + counts[q][r]] for q in range(P)])
+                for r in range(P)]
+
+    def reduce_ranges(self, tensors: Sequence[torch.Tensor], bounds: Sequence[int], op: str) -> None:
+        for r, t in enumerate(tensors):
+            lo, hi = bounds[r], bounds[r + 1]
+            acc = t[lo:hi].clone()
+            for o in tensors:
+                acc = torch.minimum(acc, o[lo:hi]) if op == "min" else torch.maximum(acc, o[lo:hi])
+            t[lo:hi] = acc
 
 
 # --------------------------------------------------------------------------- #
@@ -182,6 +258,31 @@ class CudaEngine:
         st = Stats()
         _check(lib().etg_step_end(self.g._h, ctypes.byref(st)), "etg_step_end")
         return st
+
+    # ---- push exchange (source partition, NEXT-3) ----
+    def frontier(self) -> int:
+        """Compacted active-set size of the last scan (vertices with local out-edges)."""
+        out = (ctypes.c_uint64 * 6)()
+        _check(lib().etg_debug_counters(self.g._h, out), "etg_debug_counters")
+        return int(out[1])
+
+    def push_count(self, bounds: Sequence[int], rank: int) -> List[int]:
+        P = len(bounds) - 1
+        self._bounds = torch.tensor(list(bounds), dtype=torch.int64).to(torch.int32).to(self.labels.device)
+        self._counts = torch.zeros(P, dtype=torch.int64, device=self.labels.device)
+        _check(lib().etg_push_count(self.g._h, P, rank, _ptr(self._bounds), _ptr(self._counts)), "etg_push_count")
+        return [int(x) for x in self._counts.cpu()]
+
+    def push_pack(self, counts: Sequence[int], rank: int) -> torch.Tensor:
+        P = len(counts)
+        cur = torch.tensor([sum(counts[:q]) for q in range(P)], dtype=torch.int64, device=self.labels.device)
+        pairs = torch.empty((max(sum(counts), 1), 2), dtype=torch.int32, device=self.labels.device)
+        _check(lib().etg_push_pack(self.g._h, P, rank, _ptr(self._bounds), _ptr(cur), _ptr(pairs)), "etg_push_pack")
+        return pairs[:sum(counts)]
+
+    def push_apply(self, pairs: torch.Tensor) -> None:
+        pairs = pairs.contiguous()
+        _check(lib().etg_push_apply(self.g._h, _ptr(pairs), int(pairs.shape[0])), "etg_push_apply")
 
 
 def _exchange(engines, group, alg: int, bounds: Optional[Sequence[int]] = None) -> None:
@@ -235,6 +336,69 @@ def run_partitions(engines, group, alg: int, source: int = 0, bounds: Optional[S
     return engines[0].labels, total
 
 
+def run_push(engines, group, alg: int, source: int, bounds: Sequence[int], ranks: Sequence[int],
+             mode: str = "auto"):
+    """NEXT-3: source partition + push exchange (SSSP/CC/SSWP).  Each engine
+    holds the out-edges of its owned range (``partition_csr_src``) and expands
+    only its own active vertices; labels it lowered on vertices it does not
+    own are proposals for their owners.  Per iteration, after the expand:
+      sparse -- (id, label) pairs of the moved non-owned vertices, grouped by
+                owner, one all-to-all, then atomic min/max on the receiver;
+      dense  -- element-wise min/max of the full label arrays onto each
+                owner's range (reduce-scatter);
+    ``mode="auto"`` picks whichever moves fewer bytes this iteration (8 bytes a
+    pair against 4 (P - 1) n bytes dense); all ranks agree through one sum.
+    Stops when every rank's compacted active set is empty.  ``ranks``: the rank
+    of each engine (all of 0..P-1 in loopback, [rank] under torch.distributed).
+    Returns (labels of engines[0], summed stats, {"sparse": k, "dense": k})."""
+    if alg == BFS:
+        raise EtgError("the push exchange serves SSSP/CC/SSWP; BFS uses the destination partition")
+    P = len(bounds) - 1
+    n = bounds[-1]
+    op = "max" if alg == SSWP else "min"
+    used = {"sparse": 0, "dense": 0}
+    for e in engines:
+        e.begin(alg, source)
+
+    def total(vals: List[int]) -> int:
+        t = [torch.tensor([v], dtype=torch.int64, device=e.labels.device) for v, e in zip(vals, engines)]
+        group.allreduce(t, "sum")
+        return int(t[0].item())
+
+    while total([e.frontier() for e in engines]) > 0:
+        for e in engines:
+            e.expand()
+        if P == 1:                                  # nothing is foreign
+            for e in engines:
+                e.scan()
+            continue
+        counts = [e.push_count(bounds, r) for e, r in zip(engines, ranks)]
+        pairs = total([sum(c) for c in counts])
+        sparse = mode == "sparse" or (mode == "auto" and 8 * pairs < 4 * (P - 1) * n)
+        if sparse:
+            used["sparse"] += 1
+            sends = [e.push_pack(c, r) for e, c, r in zip(engines, counts, ranks)]
+            recvs = group.alltoallv(sends, counts)
+            for e, rv in zip(engines, recvs):
+                e.push_apply(rv)
+        else:
+            used["dense"] += 1
+            labs = [e.labels for e in engines]
+            for t in labs:
+                t.bitwise_xor_(SIGN)            # uint32 order -> int32 order
+            group.reduce_ranges(labs, bounds, op)
+            for t in labs:
+                t.bitwise_xor_(SIGN)
+        for e in engines:
+            e.scan()
+    stats = [e.end() for e in engines]
+    tot = Stats()
+    tot.iterations = stats[0].iterations
+    for f in ("activations", "frontier_total", "shadows", "edges_processed"):
+        setattr(tot, f, sum(getattr(s, f) for s in stats))
+    return engines[0].labels, tot, used
+
+
 class DistGraph:
     """This rank's partition of a graph, driven over a torch.distributed group."""
 
@@ -252,3 +416,24 @@ class DistGraph:
 
     def run(self, alg: int, source: int = 0):
         return run_partitions([self.engine], self.group, alg, source, self.bounds)
+
+
+class PushDistGraph:
+    """This rank's SOURCE partition of a graph (out-edges of its owned range),
+    driven with the push exchange (``run_push``) over a torch.distributed group."""
+
+    def __init__(self, off, col, w, n: int, rank: int, world: int, *, K: int = 32, flags: int = 0,
+                 symmetric: bool = False, device="cuda", group=None, bounds=None, mode: str = "auto"):
+        from . import csr_to_device
+        self.n, self.rank, self.world, self.mode = n, rank, world, mode
+        self.bounds = bounds if bounds is not None else partition_ranges(off, col, n, world, by="out")
+        lo, hi = self.bounds[rank], self.bounds[rank + 1]
+        loff, lcol, lw = partition_csr_src(off, col, w, n, lo, hi)
+        o, c, ww, fl = csr_to_device(loff, lcol, lw, device=device)
+        self.graph = Graph(o, c, ww, n=n, K=K, flags=flags | fl, symmetric=symmetric)
+        self.engine = CudaEngine(self.graph)
+        self.group = TorchDistGroup(group)
+
+    def run(self, alg: int, source: int = 0):
+        labels, st, _ = run_push([self.engine], self.group, alg, source, self.bounds, [self.rank], self.mode)
+        return labels, st

@@ -45,11 +45,19 @@ class MockEngine:
             lab[source] = INF if alg == 3 else 0
             self._bits()[source >> 5] |= np.uint32(1 << (source & 31))
         self.st = _Stats()
+        self.snap = self._lab().copy()
         return self.scan()
 
     def scan(self):
         b = self._bits()
-        act = [v for v in range(self.n) if (int(b[v >> 5]) >> (v & 31)) & 1]
+        act = set(v for v in range(self.n) if (int(b[v >> 5]) >> (v & 31)) & 1)
+        if self.alg != 0:
+            # SSSP/CC/SSWP: also every vertex whose label moved since its snapshot
+            lab = self._lab()
+            moved = np.nonzero(lab != self.snap)[0]
+            act.update(int(v) for v in moved)
+            self.snap[moved] = lab[moved]
+        act = sorted(act)
         b[:] = 0
         self.depth += 1
         if self.alg == 0:
@@ -83,3 +91,32 @@ class MockEngine:
 
     def end(self):
         return self.st
+
+    # ---- push exchange (source partition) ----
+    def frontier(self):
+        return len(self.front)
+
+    def _moved_foreign(self, bounds, rank):
+        lab = self._lab()
+        own = np.zeros(self.n, dtype=bool)
+        own[bounds[rank]:bounds[rank + 1]] = True
+        return np.nonzero((lab != self.snap) & ~own)[0]
+
+    def push_count(self, bounds, rank):
+        mv = self._moved_foreign(bounds, rank)
+        self._pb = (list(bounds), rank)
+        return [int(((mv >= bounds[q]) & (mv < bounds[q + 1])).sum()) for q in range(len(bounds) - 1)]
+
+    def push_pack(self, counts, rank):
+        bounds, _ = self._pb
+        mv = self._moved_foreign(bounds, rank)            # ascending = grouped by owner
+        lab = self._lab()
+        pairs = np.stack([mv.astype(np.uint32), lab[mv]], axis=1) if len(mv) else np.zeros((0, 2), np.uint32)
+        self.snap[mv] = lab[mv]
+        return torch.from_numpy(pairs.astype(np.uint32).view(np.int32).reshape(-1, 2).copy())
+
+    def push_apply(self, pairs):
+        lab = self._lab()
+        pr = pairs.numpy().view(np.uint32).reshape(-1, 2)
+        for u, val in pr:
+            lab[u] = max(lab[u], val) if self.alg == 3 else min(lab[u], val)

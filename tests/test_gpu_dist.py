@@ -69,3 +69,73 @@ def test_partitioned_near_far_sssp(P, delta):
     s = gg.sample_sources(g, 1, 77 + P)[0]
     labels, st = edist.run_partitions(engines(g, P, sssp_delta=delta), edist.LoopbackGroup(), etg.SSSP, s)
     np.testing.assert_array_equal(etg.to_u32_numpy(labels), expected("sssp", g, s))
+
+
+# --------------------------------------------------------------------------- #
+# NEXT-3: source partition + push exchange (etg_push_count/pack/apply)
+# --------------------------------------------------------------------------- #
+def src_engines(g, P, K=32, flags=0):
+    bounds = edist.partition_ranges(g.off, g.col, g.n, P, by="out")
+    out = []
+    for r in range(P):
+        loff, lcol, lw = edist.partition_csr_src(g.off, g.col, g.w, g.n, bounds[r], bounds[r + 1])
+        o, c, w, fl = etg.csr_to_device(loff, lcol, lw, device="cuda")
+        G = etg.Graph(o, c, w, n=g.n, K=K, flags=flags | fl, symmetric=g.symmetric)
+        out.append(edist.CudaEngine(G))
+    return bounds, out
+
+
+def owned_labels(engs, bounds):
+    return np.concatenate([etg.to_u32_numpy(e.labels)[bounds[r]:bounds[r + 1]] for r, e in enumerate(engs)])
+
+
+@pytest.mark.parametrize("mode", ["sparse", "dense", "auto"])
+@pytest.mark.parametrize("alg", ["sssp", "cc", "sswp"])
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_push_c1(alg, P, mode):
+    g = gg.make("C1", symmetric=(alg == "cc"), weights=(alg != "cc"))
+    s = gg.sample_sources(g, 1, 11 + P)[0]
+    bounds, engs = src_engines(g, P)
+    _, st, used = edist.run_push(engs, edist.LoopbackGroup(), ALG[alg], s, bounds, list(range(P)), mode)
+    np.testing.assert_array_equal(owned_labels(engs, bounds), expected(alg, g, s))
+    if mode != "auto":
+        assert used[mode] == sum(used.values()) > 0
+
+
+def test_push_lj_small_k_and_udc_off():
+    g = gg.make("LJ-small")
+    s = gg.sample_sources(g, 1, 5)[0]
+    for K, flags in ((32, 0), (8, 0), (32, etg.NO_UDC)):
+        bounds, engs = src_engines(g, 3, K, flags)
+        edist.run_push(engs, edist.LoopbackGroup(), etg.SSSP, s, bounds, [0, 1, 2])
+        np.testing.assert_array_equal(owned_labels(engs, bounds), expected("sssp", g, s))
+
+
+def test_push_pack_pairs_are_the_moved_foreign_labels():
+    """After one expand from the source: the packed pairs are exactly the
+    vertices outside the owned range whose label the expand lowered, each once,
+    grouped by owner, with the label value."""
+    g = gg.make("C1")
+    s = gg.first_source(g)
+    P = 3
+    bounds, engs = src_engines(g, P)
+    r = next(q for q in range(P) if bounds[q] <= s < bounds[q + 1])
+    e = engs[r]
+    e.begin(etg.SSSP, s)
+    e.expand()
+    lab = etg.to_u32_numpy(e.labels).copy()
+    off, col, w = g.numpy()
+    nb = col[off[s]:off[s + 1]]
+    foreign = sorted(set(int(u) for u in nb if not (bounds[r] <= u < bounds[r + 1])))
+    counts = e.push_count(bounds, r)
+    assert counts[r] == 0 and sum(counts) == len(foreign)
+    pairs = e.push_pack(counts, r).cpu().numpy().view(np.uint32)
+    start = 0
+    for q in range(P):
+        seg = pairs[start:start + counts[q]]
+        assert all(bounds[q] <= u < bounds[q + 1] for u in seg[:, 0])
+        start += counts[q]
+    assert sorted(pairs[:, 0].tolist()) == foreign
+    assert all(lab[u] == val for u, val in pairs)
+    assert sum(e.push_count(bounds, r)) == 0            # packed = sent: snapshot refreshed
+    e.end()

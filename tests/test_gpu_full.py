@@ -45,3 +45,31 @@ def test_c3_lj_shaped(flags):
     s = gg.first_source(g)
     np.testing.assert_array_equal(U32(G.bfs(s)[0]), oracle.bfs(off, col, s))
     np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
+
+
+def test_c2_push_exchange_4way(c2):
+    """NEXT-3 at the bench size: SSSP and CC on a 4-way SOURCE partition with the
+    push exchange (auto: sparse all-to-all or dense reduce per iteration), P
+    engines on one GPU (LoopbackGroup); owned slices assembled = the oracle."""
+    from paper_conf_ipps_wangzlg19_b200 import dist as edist
+    P = 4
+
+    def run(g, alg, s):
+        bounds = edist.partition_ranges(g.off, g.col, g.n, P, by="out")
+        engs = []
+        for r in range(P):
+            loff, lcol, lw = edist.partition_csr_src(g.off, g.col, g.w, g.n, bounds[r], bounds[r + 1])
+            o, c, w, fl = etg.csr_to_device(loff, lcol, lw, device="cuda")
+            engs.append(edist.CudaEngine(etg.Graph(o, c, w, n=g.n, flags=fl, symmetric=g.symmetric)))
+        _, _, used = edist.run_push(engs, edist.LoopbackGroup(), alg, s, bounds, list(range(P)))
+        return np.concatenate([U32(e.labels)[bounds[r]:bounds[r + 1]] for r, e in enumerate(engs)]), used
+
+    off, col, w = c2.to("cpu").numpy()
+    s = gg.sample_sources(c2, 1, 4242)[0]
+    got, used = run(c2, etg.SSSP, s)
+    np.testing.assert_array_equal(got, oracle.sssp(off, col, w, s))
+    assert used["sparse"] > 0 and used["dense"] > 0          # both exchanges exercised at this size
+    gs = gg.make("C2", device="cuda", symmetric=True, weights=False)
+    soff, scol, _ = gs.to("cpu").numpy()
+    got, _ = run(gs, etg.CC, 0)
+    np.testing.assert_array_equal(got, oracle.cc(soff, scol))

@@ -1,2 +1,3 @@
-python tools/persist_diag.py --tunes 0,1024,prof 2>&1 | grep -v Warn
-ETG_LIB_PATH=paper_conf_ipps_wangzlg19_b200/libetg_sleep.so python tools/persist_diag.py --tunes 0 2>&1 | grep -v Warn
+timeout 900 python -m pytest tests/test_gpu_full.py -x -q -k push 2>&1 | tail -5
+python bench.py --partitioned --push auto --algs sssp,cc --steps 5 --warmup 3 2>&1 | tail -1
+python bench.py --partitioned --algs sssp,cc --steps 5 --warmup 3 2>&1 | tail -1
