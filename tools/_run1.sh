@@ -1,3 +1,2 @@
-timeout 900 python -m pytest tests/test_gpu_full.py -x -q -k push 2>&1 | tail -5
-python bench.py --partitioned --push auto --algs sssp,cc --steps 5 --warmup 3 2>&1 | tail -1
-python bench.py --partitioned --algs sssp,cc --steps 5 --warmup 3 2>&1 | tail -1
+timeout 900 python -m pytest tests -m "gpu and not slow" -x -q 2>&1 | tail -5
+timeout 300 bash tools/ab.sh live "ETG_TUNE=0|--algs bfs" "ETG_TUNE=2048|--algs bfs" "ETG_TUNE=0|--algs bfs" "ETG_TUNE=2048|--algs bfs"
