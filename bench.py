@@ -65,10 +65,11 @@ def parse_args():
     p.add_argument("--partitioned", action="store_true",
                    help="1-D destination partition of ONE graph over the N ranks (NCCL exchange); "
                         "default: N independent replicas")
-    p.add_argument("--push", choices=["off", "auto", "sparse", "dense"], default="off",
+    p.add_argument("--push", choices=["off", "auto", "sparse", "dense", "p2p"], default="off",
                    help="with --partitioned: SSSP/CC on a SOURCE partition with the push exchange (NEXT-3: "
-                        "all-to-all of proposals / dense reduce-scatter; auto picks per iteration); BFS keeps "
-                        "the destination partition")
+                        "all-to-all of proposals / dense reduce-scatter, auto picks per iteration; p2p: the "
+                        "expand kernel reduces into the owners' label arrays over CUDA-IPC-mapped peer "
+                        "memory); BFS keeps the destination partition")
     return p.parse_args()
 
 
@@ -583,6 +584,8 @@ def run_partitioned(args):
                     edges_tot += int(deg[lo:hi][labels[lo:hi].view(torch.int32) != -1].sum())
                 else:
                     edges_tot += int(deg[labels.view(torch.int32) != -1].sum())
+        if push:
+            dg.close()
         ms_max = allreduce([ms_tot], tdist.ReduceOp.MAX, world)[0] if world > 1 else ms_tot
         if push and a != "cc" and world > 1:
             edges_tot = int(allreduce([float(edges_tot)], tdist.ReduceOp.SUM, world)[0])

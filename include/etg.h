@@ -207,6 +207,29 @@ etg_status etg_push_count(etg_graph *g, uint32_t P, uint32_t rank, const uint32_
 etg_status etg_push_pack(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *d_bounds,
                          unsigned long long *d_cursor, uint32_t *d_pairs);
 etg_status etg_push_apply(etg_graph *g, const uint32_t *d_pairs, uint64_t count);
+
+/* Fused push exchange over peer memory (the north star's "one kernel that does
+ * both over peer memory"; replaces count/pack/all-to-all/apply).  After this
+ * call, every etg_step_expand of the handle (SSSP/CC/SSWP) applies each
+ * improving relaxation of a vertex u owned by rank q != rank (h_bounds[q] <=
+ * u < h_bounds[q+1]) twice: to its own label array (the proposal cache that
+ * filters repeats) and, as a system-scope red.min (SSWP: red.max), to
+ * h_peer_labels[q][u] -- rank q's label array, mapped into this process
+ * (etg_ipc_open of the peer's etg_ipc_handle on another GPU over NVLink, or a
+ * plain device pointer for partitions sharing a GPU).  h_peer_labels[rank] is
+ * unused.  The caller makes every rank's expand complete (stream sync + host
+ * barrier) before any rank's etg_step_scan, which then activates the owned
+ * vertices whose label moved.  h_bounds: host, P + 1 entries, 0 .. n.
+ * P = 0 turns it off.  ETG_EINVAL: P > 8, rank >= P, bad bounds, NULL
+ * pointers, or a handle without the warp expand kernel. */
+etg_status etg_push_peers(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *h_bounds,
+                          uint32_t *const *h_peer_labels);
+/* CUDA IPC for the peer label arrays: the handle (64 bytes) of the allocation
+ * holding d_ptr and d_ptr's byte offset in it; open maps a peer's handle into
+ * this process (base address; add the offset), close unmaps it. */
+etg_status etg_ipc_handle(const void *d_ptr, uint8_t *out_handle, uint64_t *out_offset);
+etg_status etg_ipc_open(const uint8_t *handle, void **out_base);
+etg_status etg_ipc_close(void *base);
 /* Tracing (step-wise runs): the device counters as of the last etg_step_* call
  * that synchronised (begin/scan/end): out[0] depth, [1] compacted active-set
  * size |F| (Proc. 1 actSet, L207), [2] shadow vertices of F (Def. 3),

@@ -94,6 +94,10 @@ def lib():
             "etg_push_count": (st, [p, u32, u32, p, p]),
             "etg_push_pack": (st, [p, u32, u32, p, p, p]),
             "etg_push_apply": (st, [p, p, u64]),
+            "etg_push_peers": (st, [p, u32, u32, p, p]),
+            "etg_ipc_handle": (st, [p, p, ctypes.POINTER(u64)]),
+            "etg_ipc_open": (st, [p, ctypes.POINTER(p)]),
+            "etg_ipc_close": (st, [p]),
             "etg_debug_expand_replay": (st, [p, ctypes.c_int, u32, u32, u32, ctypes.c_int, p, p,
                                              ctypes.POINTER(ctypes.c_float), ctypes.POINTER(u64),
                                              ctypes.POINTER(u32)]),

@@ -8,7 +8,9 @@
 // loop condition on the device, so the host synchronises once per call, not
 // once per iteration.  ETG_HOST_LOOP replaces the graph by a host loop that
 // reads the active-set size back every iteration (the paper's own control flow).
+#include <cuda.h>
 #include <cuda_runtime.h>
+#include <dlfcn.h>
 
 #include <algorithm>
 #include <atomic>
@@ -157,6 +159,9 @@ struct etg_graph {
     cudaEvent_t pev[3] = {nullptr, nullptr, nullptr};   // ETG_PROFILE: scan / expand brackets
     int step_alg = -1;                    // algorithm of the step-wise (distributed) run
     uint32_t *step_label = nullptr;       // its label array
+    uint32_t npeer = 0, peer_rank = 0;    // fused push exchange (etg_push_peers)
+    uint32_t peer_bounds[kMaxPeer + 1] = {};
+    uint32_t *peer_label[kMaxPeer] = {};
     uint64_t step_launches = 0;
     uint64_t step_acts = 0;               // activations counted so far (cumulative)
     cudaGraphExec_t exec[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -199,6 +204,10 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.ts_log2 = g->p.ts_log2;
     d.tune = g->tune;
     d.snap_used = 0;
+    d.npeer = g->npeer;
+    d.peer_rank = g->peer_rank;
+    for (uint32_t k = 0; k <= kMaxPeer; ++k) d.peer_bounds[k] = g->peer_bounds[k];
+    for (uint32_t k = 0; k < kMaxPeer; ++k) d.peer_label[k] = g->peer_label[k];
     return d;
 }
 
@@ -208,6 +217,7 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
 template <class OffT>
 Dev<OffT> make_dev_fused(const etg_graph *g, int alg) {
     Dev<OffT> d = make_dev<OffT>(g, alg);
+    d.npeer = 0;                              // the fused loop is single-partition
     d.snap_used = (alg != ALG_BFS && !(g->tune & (kTuneQMark | kTuneNoSnapUsed))) ? 1u : 0u;
     return d;
 }
@@ -222,20 +232,23 @@ const void *expand_fn(bool udc, bool idx, bool smp) {
 }
 
 template <class OffT, int ALG>
-const void *expand_warp_fn(bool udc, bool smp) {
+const void *expand_warp_fn(bool udc, bool smp, bool peer = false) {
+    if (peer && ALG != ALG_BFS)     // fused push exchange (step-wise runs only)
+        return udc ? (const void *)expand_warp_kernel<OffT, ALG, true, false, true>
+                   : (const void *)expand_warp_kernel<OffT, ALG, false, false, true>;
     if (!udc) return (const void *)expand_warp_kernel<OffT, ALG, false, false>;
     return smp ? (const void *)expand_warp_kernel<OffT, ALG, true, true>
                : (const void *)expand_warp_kernel<OffT, ALG, true, false>;
 }
 
 template <class OffT>
-const void *expand_fn_alg(int alg, bool udc, bool idx, bool smp, bool warp) {
+const void *expand_fn_alg(int alg, bool udc, bool idx, bool smp, bool warp, bool peer = false) {
     if (warp) {
         switch (alg) {
             case ALG_BFS: return expand_warp_fn<OffT, ALG_BFS>(udc, smp);
-            case ALG_SSSP: return expand_warp_fn<OffT, ALG_SSSP>(udc, smp);
-            case ALG_CC: return expand_warp_fn<OffT, ALG_CC>(udc, smp);
-            default: return expand_warp_fn<OffT, ALG_SSWP>(udc, smp);
+            case ALG_SSSP: return expand_warp_fn<OffT, ALG_SSSP>(udc, smp, peer);
+            case ALG_CC: return expand_warp_fn<OffT, ALG_CC>(udc, smp, peer);
+            default: return expand_warp_fn<OffT, ALG_SSWP>(udc, smp, peer);
         }
     }
     switch (alg) {
@@ -297,9 +310,9 @@ struct Launch {
 };
 
 template <class OffT>
-etg_status expand_launch(etg_graph *g, int alg, Launch &out) {
-    out.fn = expand_fn_alg<OffT>(alg, g->p.udc, g->p.idx, g->p.smp, g->p.warp);
-    out.smem = expand_smem(g->p, alg);
+etg_status expand_launch(etg_graph *g, int alg, Launch &out, bool peer = false) {
+    out.fn = expand_fn_alg<OffT>(alg, g->p.udc, g->p.idx, peer ? false : g->p.smp, g->p.warp, peer);
+    out.smem = peer ? 0 : expand_smem(g->p, alg);
     ETG_CU(cudaFuncSetAttribute(out.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)out.smem));
     // no dynamic shared memory: leave the unified L1/shared array to L1 (the
     // BFS visited bitmap is read through it); SMP stages: maximum shared memory
@@ -521,7 +534,8 @@ template <class OffT>
 etg_status step_expand_impl(etg_graph *g) {
     Dev<OffT> d = make_dev<OffT>(g, g->step_alg);
     Launch ex;
-    etg_status rc = expand_launch<OffT>(g, g->step_alg, ex);
+    const bool peer = g->npeer > 0 && g->step_alg != ALG_BFS;
+    etg_status rc = expand_launch<OffT>(g, g->step_alg, ex, peer);
     if (rc != ETG_OK) return rc;
     uint32_t cap_e = expand_arg(g->p);
     void *exp_args[] = {&d, &cap_e};
@@ -847,6 +861,63 @@ etg_status etg_push_apply(etg_graph *g, const uint32_t *d_pairs, uint64_t count)
         push_apply_kernel<ALG_SSSP><<<blocks, kBlock, 0, g->stream>>>(g->step_label, d_pairs, count);
     ETG_CU(cudaGetLastError());
     g->step_launches += 1;
+    return ETG_OK;
+}
+
+etg_status etg_push_peers(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *h_bounds,
+                          uint32_t *const *h_peer_labels) {
+    if (!g) return fail(ETG_EINVAL, "NULL handle");
+    if (P == 0) {
+        g->npeer = 0;
+        return ETG_OK;
+    }
+    if (!h_bounds || !h_peer_labels) return fail(ETG_EINVAL, "NULL argument");
+    if (P > kMaxPeer || rank >= P) return fail(ETG_EINVAL, "need 1 <= P <= 8 and rank < P");
+    if (!g->p.warp) return fail(ETG_EINVAL, "the fused push exchange needs the warp expand kernel");
+    if (h_bounds[0] != 0 || h_bounds[P] != g->n) return fail(ETG_EINVAL, "bounds must run from 0 to n");
+    for (uint32_t k = 0; k < P; ++k) {
+        if (h_bounds[k] > h_bounds[k + 1]) return fail(ETG_EINVAL, "bounds must be non-decreasing");
+        if (!h_peer_labels[k]) return fail(ETG_EINVAL, "NULL peer label array");
+    }
+    for (uint32_t k = 0; k <= kMaxPeer; ++k) g->peer_bounds[k] = k <= P ? h_bounds[k] : (uint32_t)g->n;
+    for (uint32_t k = 0; k < kMaxPeer; ++k) g->peer_label[k] = k < P ? h_peer_labels[k] : nullptr;
+    g->peer_rank = rank;
+    g->npeer = P;
+    return ETG_OK;
+}
+
+etg_status etg_ipc_handle(const void *d_ptr, uint8_t *out_handle, uint64_t *out_offset) {
+    if (!d_ptr || !out_handle || !out_offset) return fail(ETG_EINVAL, "NULL argument");
+    // base of the allocation holding d_ptr (driver API, resolved at run time:
+    // the library does not link libcuda)
+    typedef CUresult (*get_attr_t)(void *, CUpointer_attribute, CUdeviceptr);
+    static get_attr_t get_attr = nullptr;
+    if (!get_attr) {
+        void *h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_GLOBAL);
+        if (h) get_attr = (get_attr_t)dlsym(h, "cuPointerGetAttribute");
+        if (!get_attr) return fail(ETG_ECUDA, "cuPointerGetAttribute unavailable (no libcuda.so.1)");
+    }
+    CUdeviceptr base = 0;
+    if (get_attr(&base, CU_POINTER_ATTRIBUTE_RANGE_START_ADDR, (CUdeviceptr)d_ptr) != CUDA_SUCCESS)
+        return fail(ETG_ECUDA, "cuPointerGetAttribute(RANGE_START_ADDR) failed");
+    cudaIpcMemHandle_t hd;
+    ETG_CU(cudaIpcGetMemHandle(&hd, (void *)base));
+    memcpy(out_handle, &hd, sizeof(hd));
+    *out_offset = (uint64_t)((CUdeviceptr)d_ptr - base);
+    return ETG_OK;
+}
+
+etg_status etg_ipc_open(const uint8_t *handle, void **out_base) {
+    if (!handle || !out_base) return fail(ETG_EINVAL, "NULL argument");
+    cudaIpcMemHandle_t hd;
+    memcpy(&hd, handle, sizeof(hd));
+    ETG_CU(cudaIpcOpenMemHandle(out_base, hd, cudaIpcMemLazyEnablePeerAccess));
+    return ETG_OK;
+}
+
+etg_status etg_ipc_close(void *base) {
+    if (!base) return fail(ETG_EINVAL, "NULL argument");
+    ETG_CU(cudaIpcCloseMemHandle(base));
     return ETG_OK;
 }
 

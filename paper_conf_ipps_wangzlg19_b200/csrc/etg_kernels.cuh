@@ -92,6 +92,8 @@ struct Ctl {
     unsigned long long t_scan_ns;     //   ... and of the scan phases (block 0's view, barrier to barrier)
 };
 
+constexpr uint32_t kMaxPeer = 8;            // fused push exchange: ranks whose labels a kernel can reach
+
 template <class OffT>
 struct Dev {
     const OffT *off;
@@ -120,6 +122,14 @@ struct Dev {
     uint32_t ahead;             // warp kernel: stage A of the next batch before stage B of this one
     uint32_t nf_delta;          // near-far SSSP bucket width (0: the paper's schedule)
     uint32_t snap_used;         // SSSP/CC/SSWP, single GPU: a sole shadow stores the label it expands with
+    // Fused push exchange (NEXT-3 over peer memory): a relaxation of a vertex
+    // owned by rank q != peer_rank also lands, as a red.min/max, in rank q's
+    // label array (device memory of another GPU reached over NVLink, or of
+    // another partition on this GPU).  npeer = 0: off.
+    uint32_t npeer;
+    uint32_t peer_rank;
+    uint32_t peer_bounds[kMaxPeer + 1];
+    uint32_t *peer_label[kMaxPeer];
 };
 
 constexpr uint32_t kTuneFilterL1 = 1u;    // pre-filter label loads cached in L1
@@ -773,6 +783,32 @@ __device__ __forceinline__ void commit(uint32_t *label, uint32_t *Q, uint32_t u,
     if (ALG == ALG_BFS || markQ) red_or(&Q[u >> 5], 1u << (u & 31), pol);
 }
 
+// Fused push exchange: the local label is the proposal cache (and the
+// pre-filter's snapshot after the next scan), the owner's copy gets the same
+// reduction over peer memory.  System-scope reductions: the owner's next scan
+// runs after this kernel has completed on every rank and a host barrier.
+__device__ __forceinline__ void red_min_sys(uint32_t *p, uint32_t v) {
+    asm volatile("red.relaxed.sys.global.min.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void red_max_sys(uint32_t *p, uint32_t v) {
+    asm volatile("red.relaxed.sys.global.max.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+
+template <class OffT, int ALG>
+__device__ __forceinline__ void commit_peer(const Dev<OffT> &d, uint32_t *label, uint32_t u, uint32_t cand,
+                                            uint64_t pol) {
+    if (ALG == ALG_SSWP) red_max(&label[u], cand, pol);
+    else red_min(&label[u], cand, pol);
+    uint32_t q = 0;
+#pragma unroll
+    for (uint32_t k = 1; k < kMaxPeer; ++k)
+        q += (k < d.npeer && u >= d.peer_bounds[k]) ? 1u : 0u;
+    if (q != d.peer_rank) {
+        if (ALG == ALG_SSWP) red_max_sys(d.peer_label[q] + u, cand);
+        else red_min_sys(d.peer_label[q] + u, cand);
+    }
+}
+
 // ------------------------------------------------------------------------- //
 // A2-A5: expand.  Persistent grid; tile t covers shadows [t*ts, t*ts + ts).
 // Template switches: UDC (shadows of <= K edges, else one item per vertex),
@@ -999,7 +1035,7 @@ struct WarpTile {
     uint32_t sdelta;   // ... and stage[sdelta + x] in shared memory            (SMP)
 };
 
-template <class OffT, int ALG, bool UDC, bool SMP, bool P>
+template <class OffT, int ALG, bool UDC, bool SMP, bool P, bool PEER = false>
 __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) {
     constexpr bool kW = (ALG == ALG_SSSP || ALG == ALG_SSWP);
     constexpr uint32_t kArrays = kW ? 2u : 1u;
@@ -1257,6 +1293,12 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
                 my_passes += x;
                 return;
             }
+            if (PEER && ALG != ALG_BFS) {
+#pragma unroll
+                for (int r = 0; r < kRB; ++r)
+                    if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) commit_peer<OffT, ALG>(d, label, u[r], c[r], keep);
+                return;
+            }
 #pragma unroll
             for (int r = 0; r < kRB; ++r)
                 if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, markQ);
@@ -1386,9 +1428,9 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
     }
 }
 
-template <class OffT, int ALG, bool UDC, bool SMP>
+template <class OffT, int ALG, bool UDC, bool SMP, bool PEER = false>
 __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT> d, uint32_t capw) {
-    expand_phase<OffT, ALG, UDC, SMP, false>(d, capw);
+    expand_phase<OffT, ALG, UDC, SMP, false, PEER>(d, capw);
 }
 
 // ------------------------------------------------------------------------- //

@@ -148,6 +148,9 @@ class TorchDistGroup:
                 t[bounds[q]:bounds[q + 1]] = recv[q][:bounds[q + 1] - bounds[q]]
 
 
+    def barrier(self) -> None:
+        self.dist.barrier(group=self.group)
+
     def alltoallv(self, sends: Sequence[torch.Tensor], counts: Sequence[Sequence[int]]) -> List[torch.Tensor]:
         """sends[0]: this rank's rows (int32 [k, 2]) grouped by destination rank,
         counts[0][q] rows for rank q.  Returns [rows received, grouped by source]."""
@@ -210,6 +213,9 @@ class LoopbackGroup:
                 if t is not src:
                     t[bounds[q]:bounds[q + 1]] = src[bounds[q]:bounds[q + 1]]
 
+
+    def barrier(self) -> None:
+        pass
 
     def alltoallv(self, sends: Sequence[torch.Tensor], counts: Sequence[Sequence[int]]) -> List[torch.Tensor]:
         P = len(sends)
@@ -280,6 +286,18 @@ class CudaEngine:
         _check(lib().etg_push_pack(self.g._h, P, rank, _ptr(self._bounds), _ptr(cur), _ptr(pairs)), "etg_push_pack")
         return pairs[:sum(counts)]
 
+    def set_peers(self, bounds: Sequence[int], rank: int, peer_ptrs: Sequence[int]) -> None:
+        """Fused push exchange: relaxations of vertices owned by rank q also land
+        in peer_ptrs[q] (rank q's label array, mapped into this process)."""
+        P = len(bounds) - 1
+        b = (ctypes.c_uint32 * (P + 1))(*bounds)
+        ptrs = (ctypes.c_void_p * P)(*peer_ptrs)
+        _check(lib().etg_push_peers(self.g._h, P, rank, b, ptrs), "etg_push_peers")
+        self.peered = P > 1
+
+    def sync(self) -> None:
+        torch.cuda.synchronize(self.labels.device)
+
     def push_apply(self, pairs: torch.Tensor) -> None:
         pairs = pairs.contiguous()
         _check(lib().etg_push_apply(self.g._h, _ptr(pairs), int(pairs.shape[0])), "etg_push_apply")
@@ -336,6 +354,29 @@ def run_partitions(engines, group, alg: int, source: int = 0, bounds: Optional[S
     return engines[0].labels, total
 
 
+def open_peer_labels(engine: "CudaEngine", bounds: Sequence[int], rank: int, world: int, group=None) -> List[int]:
+    """CUDA IPC: every rank publishes the handle of its label array (all_gather_object),
+    maps every peer's into this process and registers them with the engine
+    (``set_peers``).  Returns the mapped base addresses (for etg_ipc_close)."""
+    import torch.distributed as dist
+    h = (ctypes.c_uint8 * 64)()
+    off = ctypes.c_uint64()
+    _check(lib().etg_ipc_handle(_ptr(engine.labels), h, ctypes.byref(off)), "etg_ipc_handle")
+    allh = [None] * world
+    dist.all_gather_object(allh, (bytes(h), int(off.value)), group=group)
+    ptrs, bases = [], []
+    for q, (hb, o) in enumerate(allh):
+        if q == rank:
+            ptrs.append(engine.labels.data_ptr())
+            continue
+        base = ctypes.c_void_p()
+        _check(lib().etg_ipc_open((ctypes.c_uint8 * 64)(*hb), ctypes.byref(base)), "etg_ipc_open")
+        bases.append(base.value)
+        ptrs.append(base.value + o)
+    engine.set_peers(bounds, rank, ptrs)
+    return bases
+
+
 def run_push(engines, group, alg: int, source: int, bounds: Sequence[int], ranks: Sequence[int],
              mode: str = "auto"):
     """NEXT-3: source partition + push exchange (SSSP/CC/SSWP).  Each engine
@@ -348,6 +389,10 @@ def run_push(engines, group, alg: int, source: int, bounds: Sequence[int], ranks
                 owner's range (reduce-scatter);
     ``mode="auto"`` picks whichever moves fewer bytes this iteration (8 bytes a
     pair against 4 (P - 1) n bytes dense); all ranks agree through one sum.
+    ``mode="p2p"``: the fused exchange -- the expand kernel itself applies each
+    relaxation of a foreign vertex to the owner's label array over peer memory
+    (engines set up with ``set_peers``); the host only waits for every rank's
+    expand (sync + barrier) before the scans.
     Stops when every rank's compacted active set is empty.  ``ranks``: the rank
     of each engine (all of 0..P-1 in loopback, [rank] under torch.distributed).
     Returns (labels of engines[0], summed stats, {"sparse": k, "dense": k})."""
@@ -365,9 +410,19 @@ def run_push(engines, group, alg: int, source: int, bounds: Sequence[int], ranks
         group.allreduce(t, "sum")
         return int(t[0].item())
 
+    if mode == "p2p" and P > 1 and not all(getattr(e, "peered", False) for e in engines):
+        raise EtgError("mode='p2p' needs set_peers() on every engine")
     while total([e.frontier() for e in engines]) > 0:
         for e in engines:
             e.expand()
+        if mode == "p2p" and P > 1:
+            used["p2p"] = used.get("p2p", 0) + 1
+            for e in engines:
+                e.sync()                            # this rank's remote reductions are done
+            group.barrier()                         # ... and every other rank's
+            for e in engines:
+                e.scan()
+            continue
         if P == 1:                                  # nothing is foreign
             for e in engines:
                 e.scan()
@@ -433,6 +488,14 @@ class PushDistGraph:
         self.graph = Graph(o, c, ww, n=n, K=K, flags=flags | fl, symmetric=symmetric)
         self.engine = CudaEngine(self.graph)
         self.group = TorchDistGroup(group)
+        self._ipc = []
+        if mode == "p2p" and world > 1:
+            self._ipc = open_peer_labels(self.engine, self.bounds, rank, world, group)
+
+    def close(self):
+        for base in self._ipc:
+            _check(lib().etg_ipc_close(ctypes.c_void_p(base)), "etg_ipc_close")
+        self._ipc = []
 
     def run(self, alg: int, source: int = 0):
         labels, st, _ = run_push([self.engine], self.group, alg, source, self.bounds, [self.rank], self.mode)

@@ -85,6 +85,10 @@ class MockEngine:
                 if better:
                     if self.alg != 0:
                         lab[u] = cand
+                        q = self._owner(u)
+                        if q is not None:               # fused push: the owner's copy too
+                            pl = self.peers[q]
+                            pl[u] = max(pl[u], cand) if self.alg == 3 else min(pl[u], cand)
                     self._bits()[u >> 5] |= np.uint32(1 << (u & 31))
                 self.st.edges_processed += 1
         self.st.iterations += 1
@@ -93,6 +97,23 @@ class MockEngine:
         return self.st
 
     # ---- push exchange (source partition) ----
+    peers = None
+
+    def set_peers(self, bounds, rank, peer_labels):
+        """Loopback stand-in for peer memory: the other engines' label arrays."""
+        self.pbounds, self.prank = list(bounds), rank
+        self.peers = [t.numpy().view(np.uint32) for t in peer_labels]
+        self.peered = len(bounds) > 2
+
+    def _owner(self, u):
+        if self.peers is None:
+            return None
+        q = int(np.searchsorted(np.asarray(self.pbounds), u, side="right")) - 1
+        return None if q == self.prank else q
+
+    def sync(self):
+        pass
+
     def frontier(self):
         return len(self.front)
 

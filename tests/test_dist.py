@@ -157,6 +157,29 @@ def test_push_loopback_matches_oracle(alg, P, mode):
         assert used[mode] > 0 and sum(used.values()) == used[mode]
 
 
+@pytest.mark.parametrize("alg", ["sssp", "cc", "sswp"])
+@pytest.mark.parametrize("P", [2, 3])
+def test_push_p2p_loopback_matches_oracle(alg, P):
+    """The fused exchange's driver protocol (expand writes the owners' labels,
+    sync + barrier, scan) with the numpy engine writing peers' arrays."""
+    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
+    s = gg.first_source(g)
+    bounds, parts = make_src_parts(g, P)
+    for r, p in enumerate(parts):
+        p.set_peers(bounds, r, [q.labels for q in parts])
+    _, st, used = edist.run_push(parts, edist.LoopbackGroup(), ALGS[alg], s, bounds, list(range(P)), "p2p")
+    got = owned([p.labels.numpy().view(np.uint32) for p in parts], bounds)
+    np.testing.assert_array_equal(got, expected(alg, g, s))
+    assert used.get("p2p", 0) > 0 and used["sparse"] == used["dense"] == 0
+
+
+def test_push_p2p_needs_peers():
+    g = gg.make("T12")
+    bounds, parts = make_src_parts(g, 2)
+    with pytest.raises(edist.EtgError):
+        edist.run_push(parts, edist.LoopbackGroup(), ALGS["sssp"], gg.first_source(g), bounds, [0, 1], "p2p")
+
+
 def test_push_rejects_bfs():
     g = gg.make("T12")
     bounds, parts = make_src_parts(g, 2)

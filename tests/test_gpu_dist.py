@@ -139,3 +139,68 @@ def test_push_pack_pairs_are_the_moved_foreign_labels():
     assert all(lab[u] == val for u, val in pairs)
     assert sum(e.push_count(bounds, r)) == 0            # packed = sent: snapshot refreshed
     e.end()
+
+
+# --------------------------------------------------------------------------- #
+# fused push exchange over peer memory (etg_push_peers): the expand kernel
+# writes the owners' label arrays itself
+# --------------------------------------------------------------------------- #
+@pytest.mark.parametrize("alg", ["sssp", "cc", "sswp"])
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_push_p2p_c1(alg, P):
+    g = gg.make("C1", symmetric=(alg == "cc"), weights=(alg != "cc"))
+    s = gg.sample_sources(g, 1, 31 + P)[0]
+    bounds, engs = src_engines(g, P)
+    for r, e in enumerate(engs):
+        e.set_peers(bounds, r, [x.labels.data_ptr() for x in engs])
+    _, st, used = edist.run_push(engs, edist.LoopbackGroup(), ALG[alg], s, bounds, list(range(P)), "p2p")
+    np.testing.assert_array_equal(owned_labels(engs, bounds), expected(alg, g, s))
+    assert used["p2p"] > 0 and used["sparse"] == used["dense"] == 0
+
+
+def test_push_peers_rejects_bad_arguments():
+    g = gg.make("C1")
+    bounds, engs = src_engines(g, 2)
+    e = engs[0]
+    ptrs = [x.labels.data_ptr() for x in engs]
+    for bad in ([0, 5, 7], ):                        # bounds not ending at n
+        with pytest.raises(etg.EtgError):
+            e.set_peers(bad, 0, ptrs)
+    with pytest.raises(etg.EtgError):
+        e.set_peers(bounds, 2, ptrs)                  # rank >= P
+    with pytest.raises(etg.EtgError):
+        e.set_peers([0] + [g.n] * 9, 0, [ptrs[0]] * 9)  # P = 9 > 8
+
+
+def _ipc_worker(rank, world, port, alg, out):
+    import os
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    g = gg.make("C1", symmetric=(alg == "cc"), weights=(alg != "cc"))
+    s = gg.first_source(g)
+    dg = edist.PushDistGraph(g.off, g.col, g.w, g.n, rank, world, symmetric=g.symmetric,
+                             device="cuda", mode="p2p")
+    labels, st = dg.run(ALG[alg], s)
+    lo, hi = dg.bounds[rank], dg.bounds[rank + 1]
+    np.save(out + f".{rank}.npy", etg.to_u32_numpy(labels)[lo:hi])
+    dist.barrier()
+    dg.close()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("alg", ["sssp", "cc"])
+def test_push_p2p_two_processes_cuda_ipc(alg, tmp_path):
+    """Two processes (two ranks) sharing the GPU: each maps the other's label
+    array with CUDA IPC (etg_ipc_handle/open) and its expand kernel reduces
+    into it directly -- the multi-GPU plumbing, with gloo for the host barrier."""
+    import os
+    import torch.multiprocessing as mp
+    port = 32500 + (os.getpid() % 1000) + ALG[alg]
+    out = str(tmp_path / "lab")
+    mp.spawn(_ipc_worker, args=(2, port, alg, out), nprocs=2, join=True)
+    g = gg.make("C1", symmetric=(alg == "cc"), weights=(alg != "cc"))
+    got = np.concatenate([np.load(out + f".{r}.npy") for r in range(2)])
+    np.testing.assert_array_equal(got, expected(alg, g, gg.first_source(g)))

@@ -73,3 +73,23 @@ def test_c2_push_exchange_4way(c2):
     soff, scol, _ = gs.to("cpu").numpy()
     got, _ = run(gs, etg.CC, 0)
     np.testing.assert_array_equal(got, oracle.cc(soff, scol))
+
+
+def test_c2_push_p2p_4way(c2):
+    """The fused push exchange at the bench size: 4 source partitions on one GPU,
+    each expand reducing straight into the owners' label arrays."""
+    from paper_conf_ipps_wangzlg19_b200 import dist as edist
+    P = 4
+    bounds = edist.partition_ranges(c2.off, c2.col, c2.n, P, by="out")
+    engs = []
+    for r in range(P):
+        loff, lcol, lw = edist.partition_csr_src(c2.off, c2.col, c2.w, c2.n, bounds[r], bounds[r + 1])
+        o, c, w, fl = etg.csr_to_device(loff, lcol, lw, device="cuda")
+        engs.append(edist.CudaEngine(etg.Graph(o, c, w, n=c2.n, flags=fl)))
+    for r, e in enumerate(engs):
+        e.set_peers(bounds, r, [x.labels.data_ptr() for x in engs])
+    s = gg.sample_sources(c2, 1, 4242)[0]
+    edist.run_push(engs, edist.LoopbackGroup(), etg.SSSP, s, bounds, list(range(P)), "p2p")
+    off, col, w = c2.to("cpu").numpy()
+    got = np.concatenate([U32(e.labels)[bounds[r]:bounds[r + 1]] for r, e in enumerate(engs)])
+    np.testing.assert_array_equal(got, oracle.sssp(off, col, w, s))

@@ -1,2 +1,3 @@
-timeout 900 python -m pytest tests -m "gpu and not slow" -x -q 2>&1 | tail -5
-timeout 300 bash tools/ab.sh live "ETG_TUNE=0|--algs bfs" "ETG_TUNE=2048|--algs bfs" "ETG_TUNE=0|--algs bfs" "ETG_TUNE=2048|--algs bfs"
+ab() { (cd $1 && python bench.py --steps 10 --warmup 3 --no-e2e --no-cpu-baseline --json-out /tmp/ab.json > /tmp/ab.log 2>&1; python -c "
+import json; d=json.load(open('/tmp/ab.json')); print('$1', round(d['value'],2), {k:(round(v['gteps'],1), round(v['ms_per_call'],3)) for k,v in d['per_alg'].items()})"); }
+ab _headwt; ab .; ab _headwt; ab .
