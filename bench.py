@@ -53,7 +53,10 @@ def parse_args():
     p.add_argument("--config", default="C2")
     p.add_argument("--algs", default="bfs,sssp,cc")
     p.add_argument("--K", type=int, default=32)
-    p.add_argument("--sssp-delta", type=int, default=0, help="near-far SSSP bucket width (0: paper schedule)")
+    p.add_argument("--sssp-delta", type=int, default=12,
+                   help="SSSP wave schedule: vertices at distance >= a threshold that advances by this much "
+                        "every iteration wait (0: the paper's schedule, every improved vertex every iteration); "
+                        "12 measured best on C2 (weights 1..64), DESIGN.md sec. 5")
     p.add_argument("--flags", type=int, default=0, help="extra ETG_* flags (e.g. 2 = NO_UDC)")
     p.add_argument("--sources", type=int, default=16)
     p.add_argument("--no-e2e", action="store_true")
@@ -475,7 +478,7 @@ def run_ours(args):
                 torch.cuda.synchronize()
                 ev0.record(stream)
                 etg.run_host(alg_id[a], o, c, ww, 0 if a == "cc" else s, hout, scratch, K=args.K,
-                             flags=args.flags)
+                             flags=args.flags, sssp_delta=args.sssp_delta)
                 ev1.record(stream)
                 torch.cuda.synchronize()
                 e_ms += ev0.elapsed_time(ev1)
@@ -503,6 +506,7 @@ def run_ours(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": config_desc(args.config) + "; " + "+".join(algs) + " per step",
                        "n": g.n, "m": g.m, "m_sym": m_sym, "K": args.K, "flags": args.flags,
+                       "sssp_schedule": (f"wave, Delta={args.sssp_delta}" if args.sssp_delta else "paper (Proc. 1)"),
                        "sources": len(sources),
                        "l2": "flushed (256 MiB write) before every traversal call; col/w 4 B x m each > 126 MB L2",
                        "parallelism": f"{world} independent replica(s), own sources per rank"},

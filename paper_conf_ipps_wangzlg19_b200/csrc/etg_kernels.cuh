@@ -140,6 +140,8 @@ constexpr uint32_t kTuneQMark = 64u;      // A/B: SSSP/CC/SSWP commits also set 
 constexpr uint32_t kTuneScanDyn = 256u;   // A/B: every scan tile from the counter (no static first tile)
 constexpr uint32_t kTuneNoSnapUsed = 512u; // A/B: snapshot = labels at the iteration start only
 constexpr uint32_t kTunePersist = 1024u;   // experiment: the loop as one persistent kernel (loop_kernel)
+constexpr uint32_t kTuneNoFilter = 4096u;  // A/B: no pre-filter gather, every relaxation commits
+constexpr uint32_t kTuneNearFarClassic = 8192u;   // A/B: near-far threshold advances only when the near set empties
 
 // ------------------------------------------------------------------------- //
 // small device helpers
@@ -677,6 +679,9 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                 more = true;
                 if (nF == 0) {                        // near set empty: next bucket
                     const unsigned long long thn = (unsigned long long)cld<P>(ctl->far_min) + d.nf_delta;
+                    ctl->thresh = thn > kInf ? kInf : (uint32_t)thn;
+                } else if (!(d.tune & kTuneNearFarClassic)) {   // wave: the threshold advances every iteration
+                    const unsigned long long thn = (unsigned long long)th + d.nf_delta;
                     ctl->thresh = thn > kInf ? kInf : (uint32_t)thn;
                 }
             }
@@ -1271,7 +1276,10 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
                 return;
             }
             uint32_t cur[kRB];
-            if (ALG == ALG_BFS) {
+            if (d.tune & kTuneNoFilter) {                     // A/B: every edge commits
+#pragma unroll
+                for (int r = 0; r < kRB; ++r) cur[r] = (ALG == ALG_SSWP) ? 0u : kInf;
+            } else if (ALG == ALG_BFS) {
                 // visited test on the bitmap V (n/8 bytes, read-only in this
                 // kernel, cached in L1: hits never reach the L2 request path)
 #pragma unroll

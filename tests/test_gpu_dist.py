@@ -63,8 +63,9 @@ def test_partitioned_k_and_flags():
 @pytest.mark.parametrize("P", [1, 2, 3])
 @pytest.mark.parametrize("delta", [1, 16, 1 << 20])
 def test_partitioned_near_far_sssp(P, delta):
-    """The near-far SSSP schedule through the step-wise API: deferred vertices stay in the
-    exchanged bitmap, an empty near set re-scans with the next threshold."""
+    """The near-far SSSP schedule through the step-wise API: deferred vertices keep a
+    stale snapshot (identical on every rank after the label exchange), an empty
+    near set re-scans with the next threshold."""
     g = gg.make("C1")
     s = gg.sample_sources(g, 1, 77 + P)[0]
     labels, st = edist.run_partitions(engines(g, P, sssp_delta=delta), edist.LoopbackGroup(), etg.SSSP, s)

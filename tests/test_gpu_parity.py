@@ -327,3 +327,22 @@ def test_galois_gr_file_traversal(tmp_path, c1):
     G = etg.Graph(od, cd, wd, n=c1.n, flags=fl, validate=True)
     s = gg.first_source(c1)
     np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
+
+
+@pytest.mark.parametrize("classic", [False, True])
+@pytest.mark.parametrize("delta", [3, 12, 40])
+def test_sssp_wave_and_classic_near_far(c1, delta, classic, monkeypatch):
+    """Both threshold rules of the near-far schedule: the wave (default: the
+    threshold advances by Delta every iteration) and the classic one (advance
+    only when the near set is empty; ETG_TUNE=8192).  Same distances."""
+    monkeypatch.setenv("ETG_TUNE", "8192" if classic else "0")
+    off, col, w = c1.numpy()
+    for s in gg.sample_sources(c1, 2, 100 + delta):
+        G = to_etg(c1, sssp_delta=delta)
+        d, st = G.sssp(s)
+        np.testing.assert_array_equal(U32(d), oracle.sssp(off, col, w, s))
+    g = gg.make("LJ-small", device="cuda")
+    o2, c2_, w2 = g.to("cpu").numpy()
+    s = gg.first_source(g)
+    G = to_etg(g, sssp_delta=delta)
+    np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(o2, c2_, w2, s))

@@ -64,7 +64,16 @@ if __name__ == "__main__":
     traffic = (b.get("dram__bytes_read.sum") or 0) + (b.get("dram__bytes_write.sum") or 0)
     unit = b.get("dram__bytes_read.sum [unit]", "byte")
     scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
+    # algorithmic bytes of the captured launch (BFS model: 8 B per edge + 20 B per
+    # active vertex), from the per-iteration trace of the same source
+    alg_bytes = None
+    try:
+        tr = json.load(open(f"gpurun_out/trace_{tag}.json"))["bfs"][3]
+        alg_bytes = 8 * tr["edges"] + 20 * tr["nF"]
+    except (OSError, KeyError, IndexError, ValueError):
+        pass
     summ = {"C2": {"dram_bytes_per_launch": traffic * scale,
+                   "algorithmic_bytes_of_captured_launch": alg_bytes,
                    "capture": f"profiles/ncu_{tag}.json bfs_expand_depth3 (ncu --set full, BFS depth-3 launch of C2)"}}
     json.dump(summ, open("profiles/expand_ncu_summary.json", "w"), indent=1)
     print(json.dumps(res["launch_list"], indent=1)[:1500])
