@@ -104,7 +104,7 @@ Params derive(const etg_options *opt, uint32_t tune) {
 }
 
 struct Layout {
-    size_t Q, V, snap, F, B, D, S, tile_first, recE, recS, ctl, total;
+    size_t Q, V, snap, F, B, D, S, Lx, tile_first, recE, recS, ctl, total;
     uint32_t nwords;
 };
 
@@ -129,6 +129,7 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
     L.B = take((p.u64 ? 8 : 4) * (n + 1));
     L.D = take(4 * (n + 1));
     L.S = take(4 * (n + 2));
+    L.Lx = take(4 * (n + 1));
     L.tile_first = take(4 * max_tiles);
     L.recE = take(8 * max_scan_tiles);
     L.recS = take(8 * max_scan_tiles);
@@ -186,6 +187,7 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.B = reinterpret_cast<OffT *>(g->ws + g->L.B);
     d.D = reinterpret_cast<uint32_t *>(g->ws + g->L.D);
     d.S = reinterpret_cast<uint32_t *>(g->ws + g->L.S);
+    d.Lx = reinterpret_cast<uint32_t *>(g->ws + g->L.Lx);
     d.tile_first = reinterpret_cast<uint32_t *>(g->ws + g->L.tile_first);
     d.recE = reinterpret_cast<unsigned long long *>(g->ws + g->L.recE);
     d.recS = reinterpret_cast<unsigned long long *>(g->ws + g->L.recS);
@@ -218,7 +220,12 @@ template <class OffT>
 Dev<OffT> make_dev_fused(const etg_graph *g, int alg) {
     Dev<OffT> d = make_dev<OffT>(g, alg);
     d.npeer = 0;                              // the fused loop is single-partition
-    d.snap_used = (alg != ALG_BFS && !(g->tune & (kTuneQMark | kTuneNoSnapUsed))) ? 1u : 0u;
+    // 2 = multi-shadow vertices share one published label too -- CC only:
+    // measured 1.48 -> 1.28 ms on C2; SSSP 1.96 -> 2.03 and SSWP 2.13 ->
+    // 2.17 (the compare-and-swap round trip per tile costs more than the
+    // re-expansions it saves), so they record sole shadows only
+    d.snap_used = (alg != ALG_BFS && !(g->tune & (kTuneQMark | kTuneNoSnapUsed)))
+                      ? ((alg != ALG_CC || (g->tune & kTuneNoSharedLabel)) ? 1u : 2u) : 0u;
     return d;
 }
 

@@ -106,6 +106,7 @@ struct Dev {
     OffT *B;                    // off[F[k]]
     uint32_t *D;                // out-degree of F[k] (> 0)
     uint32_t *S;                // exclusive prefix of shadow counts (nF + 1 entries)
+    uint32_t *Lx;               // snap_used: label entry k's shadows all propagate (INF = not read yet)
     uint32_t *tile_first;       // entry owning shadow t*ts
     unsigned long long *recE;   // chained scan records per scan tile: kept entries
     unsigned long long *recS;   //   and shadows (value << 32 | epoch << 2 | flag)
@@ -142,6 +143,7 @@ constexpr uint32_t kTuneNoSnapUsed = 512u; // A/B: snapshot = labels at the iter
 constexpr uint32_t kTunePersist = 1024u;   // experiment: the loop as one persistent kernel (loop_kernel)
 constexpr uint32_t kTuneNoFilter = 4096u;  // A/B: no pre-filter gather, every relaxation commits
 constexpr uint32_t kTuneNearFarClassic = 8192u;   // A/B: near-far threshold advances only when the near set empties
+constexpr uint32_t kTuneNoSharedLabel = 16384u;   // A/B: multi-shadow vertices keep the scan-time snapshot
 
 // ------------------------------------------------------------------------- //
 // small device helpers
@@ -657,6 +659,7 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                         d.B[pos] = ob[r];
                         d.D[pos] = dg;
                         d.S[pos] = sh;
+                        if (!BFSLAB && c > 1 && d.snap_used == 2u) d.Lx[pos] = kInf;   // CC: not read yet
                         // tiles whose first shadow t*ts lies in [sh, sh + c)
                         for (uint32_t t = (sh + ts - 1) >> tsl; (t << tsl) < sh + c; ++t) d.tile_first[t] = pos;
                     }
@@ -959,6 +962,7 @@ struct WarpShadow {
     OffT start;
     uint32_t len;
     uint32_t v;
+    uint32_t j;        // its entry in the compacted active set
     bool sole;         // the vertex's only shadow (its whole row)
 };
 
@@ -985,6 +989,7 @@ __device__ __forceinline__ WarpShadow<OffT, UDC> warp_map(const Dev<OffT> &d, ui
     const uint32_t sD = __shfl_sync(kFull, Dj, jj);
     WarpShadow<OffT, UDC> r;
     r.v = __shfl_sync(kFull, Fj, jj);
+    r.j = j0 + jj;
     r.len = 0;
     r.start = 0;
     r.sole = !UDC || sD <= d.K;
@@ -1185,10 +1190,22 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
         // shadow records the label it propagates in the snapshot, so the scan
         // re-activates it only if its label moves after this read (R-5).
         const bool snap_used = ALG != ALG_BFS && d.snap_used;
+        // A vertex cut into several shadows (Def. 3): the first of its shadows
+        // to start publishes the label it read in Lx (compare-and-swap on
+        // the "not read" INF), and every shadow propagates that one value, so
+        // it can be recorded in the snapshot too (snap_used == 2).
         auto src_label = [&](const WarpShadow<OffT, UDC> &sh) -> uint32_t {
             if (!sh.len) return 0u;
-            const uint32_t l = ld_cg(&label[sh.v]);
-            if (snap_used && sh.sole) d.snap[sh.v] = l;
+            uint32_t l = ld_cg(&label[sh.v]);
+            if (snap_used) {
+                if (sh.sole) {
+                    d.snap[sh.v] = l;
+                } else if (ALG == ALG_CC && d.snap_used == 2u) {
+                    const uint32_t o = atomicCAS(&d.Lx[sh.j], kInf, l);
+                    if (o != kInf) l = o;
+                    d.snap[sh.v] = l;
+                }
+            }
             return l;
         };
         uint32_t A_lab = (ALG == ALG_BFS) ? level : src_label(A_t.sh);

@@ -59,10 +59,10 @@ def test_workspace_bytes_monotone(L):
     c = L.etg_workspace_bytes(2000, 1_000_000, ctypes.byref(etg.Options(1, 0)))
     assert 0 < a < b < c
     # C2-sized workspace stays small next to the CSR (8 n B of col/w per edge x 16):
-    # snap, F, B, D, S (5 arrays of n words) + the bitmap Q + tile_first + scan descriptors
+    # snap, F, B, D, S, Lx (6 arrays of n words) + the bitmaps Q, V + tile_first + scan descriptors
     n, m = 1 << 22, 67_000_000
     ws = L.etg_workspace_bytes(n, m, ctypes.byref(o))
-    assert 20 * n < ws < 22 * n
+    assert 24 * n < ws < 26 * n
 
 
 def test_load_rejects_bad_arguments_without_gpu(L):

@@ -12,10 +12,15 @@ run c2_k16 --steps 10 --warmup 3 --K 16
 run c2_k64 --steps 10 --warmup 3 --K 64
 run c2_k256 --steps 10 --warmup 3 --K 256
 run c2_hostloop --steps 10 --warmup 3 --flags 32
-run c2_sssp_delta16 --algs sssp --steps 10 --warmup 3 --sssp-delta 16
+run c2_sssp_paper --algs sssp --steps 10 --warmup 3 --sssp-delta 0
+run c2_sssp_wave8 --algs sssp --steps 10 --warmup 3 --sssp-delta 8
+run c2_sssp_wave16 --algs sssp --steps 10 --warmup 3 --sssp-delta 16
+ETG_TUNE=8192 run c2_sssp_classic16 --algs sssp --steps 10 --warmup 3 --sssp-delta 16
 run c2_hostedges --algs bfs,sssp --steps 3 --warmup 1 --host-edges
 run c3_udc --config C3 --algs bfs,sssp --steps 10 --warmup 3
+run c3_sssp_paper --config C3 --algs sssp --steps 10 --warmup 3 --sssp-delta 0
 run c3_noudc --config C3 --algs bfs,sssp --steps 10 --warmup 3 --flags 2
 T=600 run c4_sssp --config C4 --algs sssp --steps 3 --warmup 1
+T=600 run c4_sssp_paper --config C4 --algs sssp --steps 3 --warmup 1 --sssp-delta 0
 T=600 run c4_sssp_noudc --config C4 --algs sssp --steps 2 --warmup 1 --flags 2
 T=600 run c5_bfs --config C5 --algs bfs --steps 3 --warmup 1
