@@ -144,6 +144,7 @@ constexpr uint32_t kTunePersist = 1024u;   // experiment: the loop as one persis
 constexpr uint32_t kTuneNoFilter = 4096u;  // A/B: no pre-filter gather, every relaxation commits
 constexpr uint32_t kTuneNearFarClassic = 8192u;   // A/B: near-far threshold advances only when the near set empties
 constexpr uint32_t kTuneNoSharedLabel = 16384u;   // A/B: multi-shadow vertices keep the scan-time snapshot
+constexpr uint32_t kTuneAheadAll = 32768u;        // A/B: SMP look-ahead for SSSP/CC/SSWP too (default: BFS only)
 
 // ------------------------------------------------------------------------- //
 // small device helpers
