@@ -72,7 +72,8 @@ def parse_args():
                    help="with --partitioned: SSSP/CC on a SOURCE partition with the push exchange (NEXT-3: "
                         "all-to-all of proposals / dense reduce-scatter, auto picks per iteration; p2p: the "
                         "expand kernel reduces into the owners' label arrays over CUDA-IPC-mapped peer "
-                        "memory); BFS keeps the destination partition")
+                        "memory); BFS keeps the destination partition (with p2p: owners store their new "
+                        "bitmap words straight into the peers' copies instead of the NCCL all-gather)")
     return p.parse_args()
 
 
@@ -564,7 +565,8 @@ def run_partitioned(args):
                                      symmetric=(a == "cc"), device=dev, group=group, mode=args.push)
         else:
             dg = edist.DistGraph(g.off, g.col, g.w, g.n, rank, world, K=args.K, flags=args.flags,
-                                 symmetric=(a == "cc"), device=dev, group=group)
+                                 symmetric=(a == "cc"), device=dev, group=group,
+                                 exchange="p2p" if args.push == "p2p" else "collective")
         lo, hi = dg.bounds[rank], dg.bounds[rank + 1]
         m_sym = g.m
         del g
@@ -588,7 +590,7 @@ def run_partitioned(args):
                     edges_tot += int(deg[lo:hi][labels[lo:hi].view(torch.int32) != -1].sum())
                 else:
                     edges_tot += int(deg[labels.view(torch.int32) != -1].sum())
-        if push:
+        if push or args.push == "p2p":
             dg.close()
         ms_max = allreduce([ms_tot], tdist.ReduceOp.MAX, world)[0] if world > 1 else ms_tot
         if push and a != "cc" and world > 1:

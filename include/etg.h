@@ -224,6 +224,20 @@ etg_status etg_push_apply(etg_graph *g, const uint32_t *d_pairs, uint64_t count)
  * pointers, or a handle without the warp expand kernel. */
 etg_status etg_push_peers(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *h_bounds,
                           uint32_t *const *h_peer_labels);
+/* Fused destination-partition exchange (replaces the exchange of the
+ * step-wise protocol above for destination partitions): register every
+ * rank's bitmap Q (etg_bitmap_layout) and label array, mapped into this
+ * process, and the partition bounds (host, P + 1 entries, inner bounds
+ * multiples of 32).  etg_step_publish, called after etg_step_expand, then
+ * stores what changed in this rank's owned range straight into every peer's
+ * copy: BFS -- the non-zero bitmap words (only the owner marks its vertices,
+ * so a plain store is the union); SSSP/CC/SSWP -- the labels that moved
+ * (label != snapshot).  The caller waits for every rank's publish (stream
+ * sync + host barrier) before the scans.  P = 0 turns it off; ETG_EINVAL on
+ * bad arguments, or publish without peers / outside a step-wise run. */
+etg_status etg_dest_peers(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *h_bounds,
+                          uint32_t *const *h_peer_Q, uint32_t *const *h_peer_labels);
+etg_status etg_step_publish(etg_graph *g);
 /* CUDA IPC for the peer label arrays: the handle (64 bytes) of the allocation
  * holding d_ptr and d_ptr's byte offset in it; open maps a peer's handle into
  * this process (base address; add the offset), close unmaps it. */

@@ -98,6 +98,8 @@ def lib():
             "etg_ipc_handle": (st, [p, p, ctypes.POINTER(u64)]),
             "etg_ipc_open": (st, [p, ctypes.POINTER(p)]),
             "etg_ipc_close": (st, [p]),
+            "etg_dest_peers": (st, [p, u32, u32, p, p, p]),
+            "etg_step_publish": (st, [p]),
             "etg_debug_expand_replay": (st, [p, ctypes.c_int, u32, u32, u32, ctypes.c_int, p, p,
                                              ctypes.POINTER(ctypes.c_float), ctypes.POINTER(u64),
                                              ctypes.POINTER(u32)]),

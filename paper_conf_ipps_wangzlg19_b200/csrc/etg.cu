@@ -163,6 +163,10 @@ struct etg_graph {
     uint32_t npeer = 0, peer_rank = 0;    // fused push exchange (etg_push_peers)
     uint32_t peer_bounds[kMaxPeer + 1] = {};
     uint32_t *peer_label[kMaxPeer] = {};
+    uint32_t dpeer = 0, dpeer_rank = 0;   // fused destination-partition exchange (etg_dest_peers)
+    uint32_t dpeer_lo = 0, dpeer_hi = 0;
+    uint32_t *dpeer_Q[kMaxPeer] = {};
+    uint32_t *dpeer_label[kMaxPeer] = {};
     uint64_t step_launches = 0;
     uint64_t step_acts = 0;               // activations counted so far (cumulative)
     cudaGraphExec_t exec[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -893,6 +897,54 @@ etg_status etg_push_peers(etg_graph *g, uint32_t P, uint32_t rank, const uint32_
     for (uint32_t k = 0; k < kMaxPeer; ++k) g->peer_label[k] = k < P ? h_peer_labels[k] : nullptr;
     g->peer_rank = rank;
     g->npeer = P;
+    return ETG_OK;
+}
+
+etg_status etg_dest_peers(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *h_bounds,
+                          uint32_t *const *h_peer_Q, uint32_t *const *h_peer_labels) {
+    if (!g) return fail(ETG_EINVAL, "NULL handle");
+    if (P == 0) {
+        g->dpeer = 0;
+        return ETG_OK;
+    }
+    if (!h_bounds || !h_peer_Q || !h_peer_labels) return fail(ETG_EINVAL, "NULL argument");
+    if (P > kMaxPeer || rank >= P) return fail(ETG_EINVAL, "need 1 <= P <= 8 and rank < P");
+    if (h_bounds[0] != 0 || h_bounds[P] != g->n) return fail(ETG_EINVAL, "bounds must run from 0 to n");
+    for (uint32_t k = 0; k < P; ++k) {
+        if (h_bounds[k] > h_bounds[k + 1]) return fail(ETG_EINVAL, "bounds must be non-decreasing");
+        if (k > 0 && (h_bounds[k] & 31u)) return fail(ETG_EINVAL, "inner bounds must be multiples of 32");
+        if (!h_peer_Q[k] || !h_peer_labels[k]) return fail(ETG_EINVAL, "NULL peer array");
+    }
+    for (uint32_t k = 0; k < kMaxPeer; ++k) {
+        g->dpeer_Q[k] = k < P ? h_peer_Q[k] : nullptr;
+        g->dpeer_label[k] = k < P ? h_peer_labels[k] : nullptr;
+    }
+    g->dpeer_lo = h_bounds[rank];
+    g->dpeer_hi = h_bounds[rank + 1];
+    g->dpeer_rank = rank;
+    g->dpeer = P;
+    return ETG_OK;
+}
+
+etg_status etg_step_publish(etg_graph *g) {
+    if (!g || g->step_alg < 0) return fail(ETG_EINVAL, "no step-wise run in progress");
+    if (!g->dpeer) return fail(ETG_EINVAL, "etg_dest_peers not set");
+    if (g->dpeer < 2 || g->dpeer_hi <= g->dpeer_lo) return ETG_OK;
+    PeerSet ps;
+    ps.P = g->dpeer;
+    ps.rank = g->dpeer_rank;
+    const bool bfs = g->step_alg == ALG_BFS;
+    for (uint32_t k = 0; k < kMaxPeer; ++k) ps.ptr[k] = bfs ? g->dpeer_Q[k] : g->dpeer_label[k];
+    const uint32_t *Q = reinterpret_cast<const uint32_t *>(g->ws + g->L.Q);
+    const uint32_t *snap = reinterpret_cast<const uint32_t *>(g->ws + g->L.snap);
+    if (bfs)
+        publish_kernel<true><<<g->grid_init, kBlock, 0, g->stream>>>(Q, g->step_label, snap, g->dpeer_lo,
+                                                                     g->dpeer_hi, ps);
+    else
+        publish_kernel<false><<<g->grid_init, kBlock, 0, g->stream>>>(Q, g->step_label, snap, g->dpeer_lo,
+                                                                      g->dpeer_hi, ps);
+    ETG_CU(cudaGetLastError());
+    g->step_launches += 1;
     return ETG_OK;
 }
 

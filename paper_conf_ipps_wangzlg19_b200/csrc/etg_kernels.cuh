@@ -1613,6 +1613,36 @@ __global__ __launch_bounds__(kBlock) void push_pack_kernel(const uint32_t *label
     }
 }
 
+// Fused destination-partition exchange (replaces the all-gather of owned
+// slices): the owner of [lo, hi) stores what changed in its range straight
+// into every peer's copy -- BFS: the non-zero words of its bitmap Q (no other
+// rank marks those vertices, so a plain store is the union); SSSP/CC/SSWP:
+// the labels that moved this iteration (label != snapshot).
+struct PeerSet {
+    uint32_t P, rank;
+    uint32_t *ptr[kMaxPeer];    // peer q's Q (BFS) or label array, mapped into this process
+};
+
+template <bool BFS>
+__global__ __launch_bounds__(kBlock) void publish_kernel(const uint32_t *Q, const uint32_t *label,
+                                                         const uint32_t *snap, uint32_t lo, uint32_t hi,
+                                                         PeerSet ps) {
+    const uint32_t stride = gridDim.x * blockDim.x;
+    const uint32_t a = BFS ? lo >> 5 : lo, b = BFS ? (hi + 31) >> 5 : hi;
+    for (uint32_t i = a + blockIdx.x * blockDim.x + threadIdx.x; i < b; i += stride) {
+        uint32_t x;
+        if (BFS) {
+            x = Q[i];
+            if (!x) continue;
+        } else {
+            x = __ldcg(&label[i]);
+            if (x == __ldcg(&snap[i])) continue;
+        }
+        for (uint32_t q = 0; q < ps.P; ++q)
+            if (q != ps.rank) ps.ptr[q][i] = x;
+    }
+}
+
 // Received proposals: label[id] = min(label[id], val) (SSWP: max).  The scan
 // that follows activates every owned vertex whose label moved.
 template <int ALG>

@@ -298,6 +298,20 @@ class CudaEngine:
     def sync(self) -> None:
         torch.cuda.synchronize(self.labels.device)
 
+    # ---- fused destination-partition exchange ----
+    def set_dest_peers(self, bounds: Sequence[int], rank: int, q_ptrs: Sequence[int],
+                       label_ptrs: Sequence[int]) -> None:
+        """etg_step_publish will store this rank's changes straight into the peers' copies."""
+        P = len(bounds) - 1
+        b = (ctypes.c_uint32 * (P + 1))(*bounds)
+        qp = (ctypes.c_void_p * P)(*q_ptrs)
+        lp = (ctypes.c_void_p * P)(*label_ptrs)
+        _check(lib().etg_dest_peers(self.g._h, P, rank, b, qp, lp), "etg_dest_peers")
+        self.dest_peered = True
+
+    def publish(self) -> None:
+        _check(lib().etg_step_publish(self.g._h), "etg_step_publish")
+
     def push_apply(self, pairs: torch.Tensor) -> None:
         pairs = pairs.contiguous()
         _check(lib().etg_push_apply(self.g._h, _ptr(pairs), int(pairs.shape[0])), "etg_push_apply")
@@ -332,17 +346,30 @@ def _exchange(engines, group, alg: int, bounds: Optional[Sequence[int]] = None) 
             t.bitwise_xor_(SIGN)
 
 
-def run_partitions(engines, group, alg: int, source: int = 0, bounds: Optional[Sequence[int]] = None):
+def run_partitions(engines, group, alg: int, source: int = 0, bounds: Optional[Sequence[int]] = None,
+                   exchange: str = "collective"):
     """Drive P engines in lockstep (all in this process: loopback), or ONE
     engine of this rank (torch.distributed: the other ranks run the same
     loop).  ``bounds`` (the partition, ``partition_ranges``) selects the
     all-gather exchange of owned slices; without it full arrays are
-    all-reduced.  Returns (labels of engines[0], summed stats)."""
+    all-reduced.  ``exchange="p2p"``: no collective -- each engine's
+    etg_step_publish stores its owned changes straight into the peers' copies
+    (engines set up with ``set_dest_peers``), then sync + barrier.
+    Returns (labels of engines[0], summed stats)."""
+    if exchange == "p2p" and not all(getattr(e, "dest_peered", False) for e in engines):
+        raise EtgError("exchange='p2p' needs set_dest_peers() on every engine")
     n_act = [e.begin(alg, source) for e in engines]
     while n_act[0] > 0:
         for e in engines:
             e.expand()
-        _exchange(engines, group, alg, bounds)
+        if exchange == "p2p":
+            for e in engines:
+                e.publish()
+            for e in engines:
+                e.sync()
+            group.barrier()
+        else:
+            _exchange(engines, group, alg, bounds)
         n_act = [e.scan() for e in engines]
         if len(set(n_act)) != 1:
             raise EtgError(f"ranks disagree on the active-set size: {n_act}")
@@ -354,25 +381,32 @@ def run_partitions(engines, group, alg: int, source: int = 0, bounds: Optional[S
     return engines[0].labels, total
 
 
-def open_peer_labels(engine: "CudaEngine", bounds: Sequence[int], rank: int, world: int, group=None) -> List[int]:
-    """CUDA IPC: every rank publishes the handle of its label array (all_gather_object),
-    maps every peer's into this process and registers them with the engine
-    (``set_peers``).  Returns the mapped base addresses (for etg_ipc_close)."""
+def map_peer_tensors(t: torch.Tensor, rank: int, world: int, group=None):
+    """CUDA IPC: every rank publishes the handle of its tensor t (all_gather_object)
+    and maps every peer's into this process.  Returns (device pointers of the P
+    ranks' tensors, valid in this process; mapped base addresses for etg_ipc_close)."""
     import torch.distributed as dist
     h = (ctypes.c_uint8 * 64)()
     off = ctypes.c_uint64()
-    _check(lib().etg_ipc_handle(_ptr(engine.labels), h, ctypes.byref(off)), "etg_ipc_handle")
+    _check(lib().etg_ipc_handle(_ptr(t), h, ctypes.byref(off)), "etg_ipc_handle")
     allh = [None] * world
     dist.all_gather_object(allh, (bytes(h), int(off.value)), group=group)
     ptrs, bases = [], []
     for q, (hb, o) in enumerate(allh):
         if q == rank:
-            ptrs.append(engine.labels.data_ptr())
+            ptrs.append(t.data_ptr())
             continue
         base = ctypes.c_void_p()
         _check(lib().etg_ipc_open((ctypes.c_uint8 * 64)(*hb), ctypes.byref(base)), "etg_ipc_open")
         bases.append(base.value)
         ptrs.append(base.value + o)
+    return ptrs, bases
+
+
+def open_peer_labels(engine: "CudaEngine", bounds: Sequence[int], rank: int, world: int, group=None) -> List[int]:
+    """Push exchange over peer memory: map every peer's label array and register
+    them with the engine (``set_peers``).  Returns the mapped bases."""
+    ptrs, bases = map_peer_tensors(engine.labels, rank, world, group)
     engine.set_peers(bounds, rank, ptrs)
     return bases
 
@@ -455,10 +489,12 @@ def run_push(engines, group, alg: int, source: int, bounds: Sequence[int], ranks
 
 
 class DistGraph:
-    """This rank's partition of a graph, driven over a torch.distributed group."""
+    """This rank's partition of a graph, driven over a torch.distributed group.
+    exchange="collective": all-gather of owned slices (NCCL); "p2p": each rank
+    stores its owned changes straight into the peers' copies (CUDA IPC)."""
 
     def __init__(self, off, col, w, n: int, rank: int, world: int, *, K: int = 32, flags: int = 0,
-                 symmetric: bool = False, device="cuda", group=None, bounds=None):
+                 symmetric: bool = False, device="cuda", group=None, bounds=None, exchange: str = "collective"):
         from . import csr_to_device
         self.n, self.rank, self.world = n, rank, world
         self.bounds = bounds if bounds is not None else partition_ranges(off, col, n, world)
@@ -468,9 +504,24 @@ class DistGraph:
         self.graph = Graph(o, c, ww, n=n, K=K, flags=flags | fl, symmetric=symmetric)
         self.engine = CudaEngine(self.graph)
         self.group = TorchDistGroup(group)
+        self.exchange = exchange
+        self._ipc = []
+        if exchange == "p2p":
+            if world > 1:
+                qp, qb = map_peer_tensors(self.engine.q, rank, world, group)
+                lp, lb = map_peer_tensors(self.engine.labels, rank, world, group)
+                self._ipc = qb + lb
+            else:
+                qp, lp = [self.engine.q.data_ptr()], [self.engine.labels.data_ptr()]
+            self.engine.set_dest_peers(self.bounds, rank, qp, lp)
+
+    def close(self):
+        for base in self._ipc:
+            _check(lib().etg_ipc_close(ctypes.c_void_p(base)), "etg_ipc_close")
+        self._ipc = []
 
     def run(self, alg: int, source: int = 0):
-        return run_partitions([self.engine], self.group, alg, source, self.bounds)
+        return run_partitions([self.engine], self.group, alg, source, self.bounds, self.exchange)
 
 
 class PushDistGraph:

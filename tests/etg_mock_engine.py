@@ -141,3 +141,26 @@ class MockEngine:
         pr = pairs.numpy().view(np.uint32).reshape(-1, 2)
         for u, val in pr:
             lab[u] = max(lab[u], val) if self.alg == 3 else min(lab[u], val)
+
+    # ---- fused destination-partition exchange ----
+    def set_dest_peers(self, bounds, rank, peer_q, peer_labels):
+        """Loopback stand-in for peer memory: the other engines' bitmap / label tensors."""
+        self.dbounds, self.drank = list(bounds), rank
+        self.dpeer_q = [t.numpy().view(np.uint32) for t in peer_q]
+        self.dpeer_l = [t.numpy().view(np.uint32) for t in peer_labels]
+        self.dest_peered = True
+
+    def publish(self):
+        lo, hi = self.dbounds[self.drank], self.dbounds[self.drank + 1]
+        for q in range(len(self.dbounds) - 1):
+            if q == self.drank:
+                continue
+            if self.alg == 0:
+                a, b = lo >> 5, (hi + 31) >> 5
+                src = self._bits()[a:b]
+                nz = np.nonzero(src)[0]
+                self.dpeer_q[q][a + nz] = src[nz]
+            else:
+                lab = self._lab()
+                mv = np.nonzero(lab[lo:hi] != self.snap[lo:hi])[0] + lo
+                self.dpeer_l[q][mv] = lab[mv]

@@ -76,6 +76,21 @@ def test_loopback_driver_matches_oracle(alg, P, gather):
         assert st.edges_processed == int(np.diff(g.off.numpy())[expected(alg, g, s) != oracle.INF].sum())
 
 
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "cc", "sswp"])
+@pytest.mark.parametrize("P", [2, 3])
+def test_dest_p2p_loopback_matches_oracle(alg, P):
+    """The fused destination-partition exchange's protocol: each engine
+    publishes its owned changes into the peers' copies, no collective."""
+    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
+    s = gg.first_source(g)
+    bounds, parts = make_parts(g, P)
+    for r, p in enumerate(parts):
+        p.set_dest_peers(bounds, r, [q.q for q in parts], [q.labels for q in parts])
+    labels, st = edist.run_partitions(parts, edist.LoopbackGroup(), ALGS[alg], s, bounds, "p2p")
+    for p in parts:       # every rank holds the full result, as with the all-gather
+        np.testing.assert_array_equal(p.labels.numpy().view(np.uint32), expected(alg, g, s))
+
+
 def _gloo_worker(rank, world, port, alg, out, gather=False):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)

@@ -205,3 +205,67 @@ def test_push_p2p_two_processes_cuda_ipc(alg, tmp_path):
     g = gg.make("C1", symmetric=(alg == "cc"), weights=(alg != "cc"))
     got = np.concatenate([np.load(out + f".{r}.npy") for r in range(2)])
     np.testing.assert_array_equal(got, expected(alg, g, gg.first_source(g)))
+
+
+# --------------------------------------------------------------------------- #
+# fused destination-partition exchange (etg_dest_peers / etg_step_publish):
+# owners store their changes straight into the peers' copies, no collective
+# --------------------------------------------------------------------------- #
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "cc", "sswp"])
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_dest_p2p_c1(alg, P):
+    g = gg.make("C1", symmetric=(alg == "cc"), weights=(alg != "cc"))
+    s = gg.sample_sources(g, 1, 51 + P)[0]
+    engs = engines(g, P)
+    bounds = edist.partition_ranges(g.off, g.col, g.n, P)
+    for r, e in enumerate(engs):
+        e.set_dest_peers(bounds, r, [x.q.data_ptr() for x in engs], [x.labels.data_ptr() for x in engs])
+    labels, st = edist.run_partitions(engs, edist.LoopbackGroup(), ALG[alg], s, bounds, "p2p")
+    exp = expected(alg, g, s)
+    for e in engs:
+        np.testing.assert_array_equal(etg.to_u32_numpy(e.labels), exp)
+
+
+def test_dest_p2p_near_far_sssp():
+    g = gg.make("C1")
+    s = gg.sample_sources(g, 1, 5)[0]
+    P = 3
+    engs = engines(g, P, sssp_delta=16)
+    bounds = edist.partition_ranges(g.off, g.col, g.n, P)
+    for r, e in enumerate(engs):
+        e.set_dest_peers(bounds, r, [x.q.data_ptr() for x in engs], [x.labels.data_ptr() for x in engs])
+    labels, _ = edist.run_partitions(engs, edist.LoopbackGroup(), etg.SSSP, s, bounds, "p2p")
+    np.testing.assert_array_equal(etg.to_u32_numpy(labels), expected("sssp", g, s))
+
+
+def _ipc_dest_worker(rank, world, port, alg, out):
+    import os
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    g = gg.make("C1", symmetric=(alg == "cc"), weights=(alg != "cc"))
+    s = gg.first_source(g)
+    dg = edist.DistGraph(g.off, g.col, g.w, g.n, rank, world, symmetric=g.symmetric, device="cuda",
+                         exchange="p2p")
+    labels, st = dg.run(ALG[alg], s)
+    np.save(out + f".{rank}.npy", etg.to_u32_numpy(labels))
+    dist.barrier()
+    dg.close()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("alg", ["bfs", "sssp"])
+def test_dest_p2p_two_processes_cuda_ipc(alg, tmp_path):
+    """Two ranks in two processes sharing the GPU: each maps the other's bitmap
+    and label array over CUDA IPC and publishes its owned changes into them."""
+    import os
+    import torch.multiprocessing as mp
+    port = 33500 + (os.getpid() % 1000) + ALG[alg]
+    out = str(tmp_path / "lab")
+    mp.spawn(_ipc_dest_worker, args=(2, port, alg, out), nprocs=2, join=True)
+    g = gg.make("C1", symmetric=(alg == "cc"), weights=(alg != "cc"))
+    exp = expected(alg, g, gg.first_source(g))
+    for r in range(2):
+        np.testing.assert_array_equal(np.load(out + f".{r}.npy"), exp)
