@@ -269,3 +269,27 @@ def test_dest_p2p_two_processes_cuda_ipc(alg, tmp_path):
     exp = expected(alg, g, gg.first_source(g))
     for r in range(2):
         np.testing.assert_array_equal(np.load(out + f".{r}.npy"), exp)
+
+
+def test_exchange_entry_points_reject_misuse():
+    """Error paths of the NEXT-3 / peer-memory entry points (ETG_EINVAL, no crash)."""
+    g = gg.make("C1")
+    bounds, engs = src_engines(g, 2)
+    e = engs[0]
+    # push entries outside an SSSP/CC/SSWP step-wise run
+    with pytest.raises(etg.EtgError):
+        e.push_count(bounds, 0)
+    e.begin(etg.BFS, gg.first_source(g))
+    with pytest.raises(etg.EtgError):
+        e.push_count(bounds, 0)                       # BFS keeps the destination partition
+    with pytest.raises(etg.EtgError):
+        e.publish()                                   # no etg_dest_peers
+    e.end()
+    qp = [x.q.data_ptr() for x in engs]
+    lp = [x.labels.data_ptr() for x in engs]
+    with pytest.raises(etg.EtgError):
+        e.set_dest_peers([0, 33, g.n], 0, qp, lp)     # inner bound not a multiple of 32
+    with pytest.raises(etg.EtgError):
+        e.set_dest_peers([0, 64, g.n], 2, qp, lp)     # rank >= P
+    with pytest.raises(etg.EtgError):
+        e.set_dest_peers([0, 64, g.n - 1], 0, qp, lp) # bounds must end at n

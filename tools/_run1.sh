@@ -1,3 +1,1 @@
-timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
-bash tools/profile_round.sh r01
-bash tools/evidence.sh 2>&1
+timeout 900 python -m pytest tests -m "gpu and not slow" -x -q 2>&1 | tail -4
