@@ -258,7 +258,12 @@ void etg_free(etg_graph *g);
  * execution).  alg: 0 = BFS, 1 = SSSP, 2 = CC, 3 = SSWP.  Copies the CSR
  * host->device into d_scratch (caller-owned device memory of at least
  * etg_host_scratch_bytes), runs the traversal and copies the n labels back into
- * h_labels.  Host buffers should be pinned for full PCIe bandwidth. */
+ * h_labels.  Host buffers should be pinned for full PCIe bandwidth.  The
+ * internal handle over d_scratch is kept per calling thread (up to 4) and
+ * reused by a later call with the same n, m, weights, scratch, stream and
+ * options (its device state is re-zeroed; nothing is read from the previous
+ * call), so only the first call pays the host-side setup.  Not re-entrant
+ * across threads sharing one scratch buffer. */
 size_t etg_host_scratch_bytes(uint64_t n, uint64_t m, int has_weights, const etg_options *opt);
 etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_row_offsets,
                         const uint32_t *h_col_idx, const uint32_t *h_weights,
