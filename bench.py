@@ -53,10 +53,11 @@ def parse_args():
     p.add_argument("--config", default="C2")
     p.add_argument("--algs", default="bfs,sssp,cc")
     p.add_argument("--K", type=int, default=32)
-    p.add_argument("--sssp-delta", type=int, default=12,
+    p.add_argument("--sssp-delta", default="auto",
                    help="SSSP wave schedule: vertices at distance >= a threshold that advances by this much "
-                        "every iteration wait (0: the paper's schedule, every improved vertex every iteration); "
-                        "12 measured best on C2 (weights 1..64), DESIGN.md sec. 5")
+                        "every iteration wait (0: the paper's schedule, every improved vertex every iteration; "
+                        "auto: 3/8 of the mean edge weight = 12 for the configs' 1..64 weights, the value "
+                        "measured best on C2), DESIGN.md sec. 5")
     p.add_argument("--flags", type=int, default=0, help="extra ETG_* flags (e.g. 2 = NO_UDC)")
     p.add_argument("--sources", type=int, default=16)
     p.add_argument("--no-e2e", action="store_true")
@@ -507,7 +508,8 @@ def run_ours(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": config_desc(args.config) + "; " + "+".join(algs) + " per step",
                        "n": g.n, "m": g.m, "m_sym": m_sym, "K": args.K, "flags": args.flags,
-                       "sssp_schedule": (f"wave, Delta={args.sssp_delta}" if args.sssp_delta else "paper (Proc. 1)"),
+                       "sssp_schedule": (f"wave, Delta={args.sssp_delta}" if str(args.sssp_delta) != "0"
+                                         else "paper (Proc. 1)"),
                        "sources": len(sources),
                        "l2": "flushed (256 MiB write) before every traversal call; col/w 4 B x m each > 126 MB L2",
                        "parallelism": f"{world} independent replica(s), own sources per rank"},

@@ -81,13 +81,17 @@ typedef struct {
     uint32_t degree_limit_k; /* K of Def. 3; 0 -> default 32 */
     uint32_t flags;          /* ETG_* bits above */
     uint32_t sssp_delta;     /* 0: the paper's schedule (every improved vertex is active in the
-                                next iteration, L64/L78).  > 0: near-far schedule for SSSP --
+                                next iteration, L64/L78).  > 0: wave schedule for SSSP --
                                 improved vertices at distance >= a threshold stay active but are
-                                deferred; the threshold advances by sssp_delta when no nearer
-                                vertex is active.  Same distances (unique fixpoint), fewer
-                                redundant relaxations.  The step-wise (multi-GPU) API honours it
-                                too: the deferred vertices stay in the exchanged bitmap. */
+                                deferred; the threshold advances by sssp_delta after every
+                                iteration (and jumps past an empty gap).  Same distances (unique
+                                fixpoint), fewer redundant relaxations.  ETG_SSSP_DELTA_AUTO:
+                                3/8 of the mean edge weight (one O(m) reduction at the first SSSP
+                                call of the handle; 12 for the 1..64 weights of the configs).
+                                The step-wise (multi-GPU) API honours it too: the deferred
+                                vertices keep a stale snapshot, identical on every rank. */
 } etg_options;
+#define ETG_SSSP_DELTA_AUTO 0xFFFFFFFFu
 
 typedef struct {
     uint32_t iterations;       /* non-empty active sets processed (Proc. 1 while-loop trips) */

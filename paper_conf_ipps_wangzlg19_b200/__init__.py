@@ -112,6 +112,14 @@ def lib():
     return _lib
 
 
+SSSP_DELTA_AUTO = 0xFFFFFFFF
+
+
+def _delta(d) -> int:
+    """sssp_delta: an int (0 = the paper's schedule) or "auto" (3/8 of the mean weight)."""
+    return SSSP_DELTA_AUTO if d == "auto" else int(d)
+
+
 def _check(rc: int, what: str):
     if rc != 0:
         L = lib()
@@ -197,7 +205,7 @@ class Graph:
             raise EtgError("row offsets must live on the device")
         self._keep = (off, col, w)
         self._stream = stream
-        self._opt = Options(K, flags, sssp_delta)
+        self._opt = Options(K, flags, _delta(sssp_delta))
         L = lib()
         nbytes = L.etg_workspace_bytes(self.n, self.m, ctypes.byref(self._opt))
         self.workspace = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=self.device)
@@ -321,7 +329,7 @@ def run_host(alg: int, off: torch.Tensor, col: torch.Tensor, w: Optional[torch.T
         flags |= SYMMETRIC
     n = int(off.shape[0] - 1)
     m = int(col.shape[0])
-    opt = Options(K, flags, sssp_delta)
+    opt = Options(K, flags, _delta(sssp_delta))
     st = Stats()
     rc = lib().etg_run_host(alg, n, m, _ptr(off), _ptr(col), _ptr(w), source, _ptr(labels_out),
                             _ptr(scratch), scratch.numel() * scratch.element_size(),

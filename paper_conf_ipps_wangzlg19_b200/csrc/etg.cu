@@ -558,10 +558,32 @@ etg_status step_expand_impl(etg_graph *g) {
     return ETG_OK;
 }
 
+// ETG_SSSP_DELTA_AUTO: Delta = 3/8 of the mean edge weight (>= 1), resolved once per handle.
+etg_status resolve_delta(etg_graph *g) {
+    if (g->p.nf_delta != ETG_SSSP_DELTA_AUTO) return ETG_OK;
+    uint32_t delta = 1;
+    if (g->m && g->w) {
+        ETG_CU(cudaMemsetAsync(&g->ctl->reached_e, 0, sizeof(unsigned long long), g->stream));
+        weight_sum_kernel<<<g->grid_init, kBlock, 0, g->stream>>>(g->w, g->m, g->ctl);
+        ETG_CU(cudaGetLastError());
+        ETG_CU(cudaMemcpyAsync(&g->h_ctl->reached_e, &g->ctl->reached_e, sizeof(unsigned long long),
+                               cudaMemcpyDeviceToHost, g->stream));
+        ETG_CU(cudaStreamSynchronize(g->stream));
+        const unsigned long long d = g->h_ctl->reached_e * 3ull / (8ull * g->m);
+        delta = d < 1 ? 1u : (d > 0x7FFFFFFFull ? 0x7FFFFFFFu : (uint32_t)d);
+    }
+    g->p.nf_delta = delta;
+    return ETG_OK;
+}
+
 etg_status run(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stats *st) {
     if (!g || !label) return fail(ETG_EINVAL, "null handle or label pointer");
     if (alg != ALG_CC && source >= g->n) return fail(ETG_EINVAL, "source >= n");
     if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "graph loaded without weights");
+    if (alg == ALG_SSSP) {
+        etg_status rc = resolve_delta(g);
+        if (rc != ETG_OK) return rc;
+    }
     if (alg == ALG_CC && !(g->flags & ETG_SYMMETRIC)) return fail(ETG_ENOTSYM, "etg_cc needs ETG_SYMMETRIC");
     if (g->n == 0) return ETG_OK;
     return g->p.u64 ? run_impl<uint64_t>(g, alg, source, label, st)
@@ -801,6 +823,8 @@ etg_status etg_step_begin(etg_graph *g, int alg, uint32_t source, uint32_t *d_la
     if (alg != ALG_CC && source >= g->n) return fail(ETG_EINVAL, "source >= n");
     if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "graph loaded without weights");
     if (alg == ALG_CC && !(g->flags & ETG_SYMMETRIC)) return fail(ETG_ENOTSYM, "etg_cc needs ETG_SYMMETRIC");
+    if (alg == ALG_SSSP && g->p.nf_delta == ETG_SSSP_DELTA_AUTO)   // ranks hold different edges
+        return fail(ETG_EINVAL, "step-wise runs need an explicit sssp_delta (every rank the same)");
     if (g->n == 0) { *n_active = 0; return ETG_OK; }
     return g->p.u64 ? step_begin_impl<uint64_t>(g, alg, source, d_label, n_active, 0)
                     : step_begin_impl<uint32_t>(g, alg, source, d_label, n_active, 0);

@@ -1660,6 +1660,16 @@ __global__ __launch_bounds__(kBlock) void push_apply_kernel(uint32_t *label, con
 // ------------------------------------------------------------------------- //
 // statistics and validation
 // ------------------------------------------------------------------------- //
+// Sum of the edge weights (ETG_SSSP_DELTA_AUTO) into ctl->reached_e.
+__global__ __launch_bounds__(kBlock) void weight_sum_kernel(const uint32_t *w, unsigned long long m, Ctl *ctl) {
+    unsigned long long acc = 0;
+    for (unsigned long long e = blockIdx.x * (unsigned long long)kBlock + threadIdx.x; e < m;
+         e += (unsigned long long)gridDim.x * kBlock)
+        acc += __ldcs(&w[e]);
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(kFull, acc, o);
+    if (lane_id() == 0 && acc) atomicAdd(&ctl->reached_e, acc);
+}
+
 template <class OffT>
 __global__ __launch_bounds__(kBlock) void reach_kernel(Dev<OffT> d, const uint32_t *label,
                                                         uint32_t unreached) {

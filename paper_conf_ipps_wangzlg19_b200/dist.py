@@ -354,11 +354,15 @@ def run_partitions(engines, group, alg: int, source: int = 0, bounds: Optional[S
     all-gather exchange of owned slices; without it full arrays are
     all-reduced.  ``exchange="p2p"``: no collective -- each engine's
     etg_step_publish stores its owned changes straight into the peers' copies
-    (engines set up with ``set_dest_peers``), then sync + barrier.
+    (engines set up with ``set_dest_peers``), then sync + barrier; barriers
+    after the initialisation and after the scans keep a rank's stores out of a
+    peer's copy until that peer has initialised it / finished scanning it.
     Returns (labels of engines[0], summed stats)."""
     if exchange == "p2p" and not all(getattr(e, "dest_peered", False) for e in engines):
         raise EtgError("exchange='p2p' needs set_dest_peers() on every engine")
     n_act = [e.begin(alg, source) for e in engines]
+    if exchange == "p2p":
+        group.barrier()     # every peer has initialised its copies before anyone publishes
     while n_act[0] > 0:
         for e in engines:
             e.expand()
@@ -371,6 +375,9 @@ def run_partitions(engines, group, alg: int, source: int = 0, bounds: Optional[S
         else:
             _exchange(engines, group, alg, bounds)
         n_act = [e.scan() for e in engines]
+        if exchange == "p2p":
+            # nobody publishes iteration k+1 into a peer still scanning iteration k
+            group.barrier()
         if len(set(n_act)) != 1:
             raise EtgError(f"ranks disagree on the active-set size: {n_act}")
     stats = [e.end() for e in engines]

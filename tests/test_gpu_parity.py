@@ -346,3 +346,21 @@ def test_sssp_wave_and_classic_near_far(c1, delta, classic, monkeypatch):
     s = gg.first_source(g)
     G = to_etg(g, sssp_delta=delta)
     np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(o2, c2_, w2, s))
+
+
+def test_sssp_delta_auto(c1):
+    """ETG_SSSP_DELTA_AUTO: Delta from the mean weight, same distances; the
+    step-wise API refuses it (ranks would each derive their own Delta)."""
+    off, col, w = c1.numpy()
+    G = to_etg(c1, sssp_delta="auto")
+    for s in gg.sample_sources(c1, 2, 77):
+        np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
+    from paper_conf_ipps_wangzlg19_b200 import dist as edist
+    e = edist.CudaEngine(to_etg(c1, sssp_delta="auto"))   # fresh handle: Delta not resolved yet
+    with pytest.raises(etg.EtgError):
+        e.begin(etg.SSSP, 0)
+    # weights all 1: Delta = max(1, 3/8) = 1, the wave then advances one hop per iteration
+    g1 = gg.Graph("unit", c1.n, c1.off, c1.col, torch.ones_like(c1.w))
+    o1, c1_, w1 = g1.numpy()
+    s = gg.first_source(c1)
+    np.testing.assert_array_equal(U32(to_etg(g1, sssp_delta="auto").sssp(s)[0]), oracle.bfs(o1, c1_, s))

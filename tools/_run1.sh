@@ -1,3 +1,2 @@
+for i in 1 2 3 4 5; do timeout 300 python -m pytest tests/test_gpu_dist.py -x -q -k "two_processes" 2>&1 | tail -1; done
 timeout 900 python -m pytest tests -m "gpu and not slow" -x -q 2>&1 | tail -3
-python tools/e2e_diag.py 0 2>&1 | grep run_host
-python bench.py --steps 10 --warmup 3 --no-cpu-baseline 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(d['value'], d['e2e'])"
