@@ -1443,6 +1443,7 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
 #endif
     // statistics: one global atomic per CTA (per-warp partials in shared memory)
     __shared__ unsigned long long s_edges;
+    __syncwarp();                                         // reconverge before the block barrier
     if (threadIdx.x == 0) s_edges = 0;
     __syncthreads();
     if (lane == 0 && my_edges) atomicAdd(&s_edges, my_edges);
