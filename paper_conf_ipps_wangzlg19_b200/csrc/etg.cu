@@ -408,8 +408,6 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
         if (rc != ETG_OK) return rc;
     }
     ETG_CU(cudaEventRecord(g->ev0, s));
-    ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, label, source);
-    if (d.nf_delta) ctl_nearfar_kernel<<<1, 1, 0, s>>>(g->ctl, d.nf_delta);
     {
         void *args[] = {&d, &label, &source};
         ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), args, 0, s));
@@ -419,7 +417,7 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
     void *scan_args[] = {&d, &none, &zero};
     // A2 of the initial active set (Proc. 1 "Init actSet")
     ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
-    uint64_t launches = 3;
+    uint64_t launches = 2;                       // init (+ control block), first scan
     if (persist) {
         // the whole loop in one cooperative launch (all CTAs co-resident)
         const void *fn = loop_fn<OffT>(alg, g->p.udc);
@@ -502,11 +500,9 @@ etg_status step_begin_impl(etg_graph *g, int alg, uint32_t source, uint32_t *lab
                            int skip_scan) {
     Dev<OffT> d = make_dev<OffT>(g, alg);
     cudaStream_t s = g->stream;
-    ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, label, source);
-    if (d.nf_delta) ctl_nearfar_kernel<<<1, 1, 0, s>>>(g->ctl, d.nf_delta);
     void *iargs[] = {&d, &label, &source};
     ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), iargs, 0, s));
-    g->step_launches = 2;
+    g->step_launches = 1;
     g->step_alg = alg;
     g->step_label = label;
     g->step_acts = 0;

@@ -299,7 +299,7 @@ __device__ __forceinline__ uint32_t udc_count(D deg, uint32_t K, uint32_t klog) 
 // A1: per-call control reset and label initialisation (Proc. 1 "Init label",
 // "Init actSet", L207)
 // ------------------------------------------------------------------------- //
-__global__ void ctl_begin_kernel(Ctl *ctl, uint32_t *label, uint32_t source) {
+__device__ __forceinline__ void ctl_begin(Ctl *ctl, uint32_t *label, uint32_t source, uint32_t thresh) {
     ctl->depth = kInf;            // the first scan makes it 0
     ctl->epoch += 1;
     ctl->nF = 0;
@@ -313,7 +313,7 @@ __global__ void ctl_begin_kernel(Ctl *ctl, uint32_t *label, uint32_t source) {
     ctl->frontier = 0;
     ctl->label = label;
     ctl->source = source;
-    ctl->thresh = 0xFFFFFFFFu;
+    ctl->thresh = thresh;         // near-far SSSP: the first threshold (the source has distance 0)
     ctl->far_min = 0xFFFFFFFFu;
     ctl->far_count = 0;
     ctl->bar = 0;
@@ -321,8 +321,9 @@ __global__ void ctl_begin_kernel(Ctl *ctl, uint32_t *label, uint32_t source) {
     ctl->t_scan_ns = 0;
 }
 
-// near-far SSSP: the first threshold (the source has distance 0)
-__global__ void ctl_nearfar_kernel(Ctl *ctl, uint32_t delta) { ctl->thresh = delta; }
+__global__ void ctl_begin_kernel(Ctl *ctl, uint32_t *label, uint32_t source) {
+    ctl_begin(ctl, label, source, kInf);
+}
 
 // the scan bookkeeping an expand launch does (see expand kernels), for a scan
 // that directly follows another scan (step-wise near-far: empty near set)
@@ -338,6 +339,8 @@ __global__ void ctl_rescan_kernel(Ctl *ctl) {
 // ones).  Q is all-zero on entry (every scan clears what it reads).
 template <class OffT, int ALG>
 __global__ __launch_bounds__(kBlock) void init_kernel(Dev<OffT> d, uint32_t *label, uint32_t source) {
+    // the control block of the call (one thread; the first scan is stream-ordered after this kernel)
+    if (blockIdx.x == 0 && threadIdx.x == 0) ctl_begin(d.ctl, label, source, d.nf_delta ? d.nf_delta : kInf);
     const uint32_t n = d.n;
     const uint32_t stride = gridDim.x * kBlock;
     for (uint32_t v = blockIdx.x * kBlock + threadIdx.x; v < n; v += stride) {
