@@ -232,7 +232,8 @@ Dev<OffT> make_dev_fused(const etg_graph *g, int alg) {
     // 2.17 (the compare-and-swap round trip per tile costs more than the
     // re-expansions it saves), so they record sole shadows only
     d.snap_used = (alg != ALG_BFS && !(g->tune & (kTuneQMark | kTuneNoSnapUsed)))
-                      ? ((alg != ALG_CC || (g->tune & kTuneNoSharedLabel)) ? 1u : 2u) : 0u;
+                      ? (((alg != ALG_CC && !(ETG_SHARED_SSSP && alg == ALG_SSSP)) || (g->tune & kTuneNoSharedLabel))
+                             ? 1u : 2u) : 0u;
     return d;
 }
 

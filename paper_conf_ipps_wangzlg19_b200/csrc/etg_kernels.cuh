@@ -51,6 +51,9 @@ constexpr uint32_t kFull = 0xFFFFFFFFu;
 #ifndef ETG_SGRAB
 #define ETG_SGRAB 1                         // expand: first tile grab static (global warp index)
 #endif
+#ifndef ETG_SHARED_SSSP
+#define ETG_SHARED_SSSP 0                   // experiment: SSSP multi-shadow vertices share one published label too
+#endif
 #ifndef ETG_BAR_SLEEP
 #define ETG_BAR_SLEEP 0                     // persistent loop: ns of back-off per grid-barrier poll
 #endif
@@ -1204,7 +1207,7 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
             if (snap_used) {
                 if (sh.sole) {
                     d.snap[sh.v] = l;
-                } else if (ALG == ALG_CC && d.snap_used == 2u) {
+                } else if ((ALG == ALG_CC || (ETG_SHARED_SSSP && ALG == ALG_SSSP)) && d.snap_used == 2u) {
                     const uint32_t o = atomicCAS(&d.Lx[sh.j], kInf, l);
                     if (o != kInf) l = o;
                     d.snap[sh.v] = l;
