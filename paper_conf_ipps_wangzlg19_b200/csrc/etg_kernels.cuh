@@ -51,6 +51,9 @@ constexpr uint32_t kFull = 0xFFFFFFFFu;
 #ifndef ETG_SGRAB
 #define ETG_SGRAB 1                         // expand: first tile grab static (global warp index)
 #endif
+#ifndef ETG_LX_PEEK
+#define ETG_LX_PEEK 1                       // shared shadow label: plain load before the compare-and-swap
+#endif
 #ifndef ETG_SHARED_SSSP
 #define ETG_SHARED_SSSP 0                   // experiment: SSSP multi-shadow vertices share one published label too
 #endif
@@ -1208,7 +1211,14 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
                 if (sh.sole) {
                     d.snap[sh.v] = l;
                 } else if ((ALG == ALG_CC || (ETG_SHARED_SSSP && ALG == ALG_SSSP)) && d.snap_used == 2u) {
+#if ETG_LX_PEEK
+                    // published already? (a plain load: hubs of many shadows do not
+                    // serialise on one compare-and-swap)
+                    uint32_t o = ld_cg(&d.Lx[sh.j]);
+                    if (o == kInf) o = atomicCAS(&d.Lx[sh.j], kInf, l);
+#else
                     const uint32_t o = atomicCAS(&d.Lx[sh.j], kInf, l);
+#endif
                     if (o != kInf) l = o;
                     d.snap[sh.v] = l;
                 }
