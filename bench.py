@@ -377,6 +377,7 @@ def run_ours(args):
                 acc[a]["ms"] += ms
                 acc[a]["edges"] += edges
                 acc[a]["calls"] += 1
+                acc[a]["rates"].append(edges / ms / 1e6)
 
     for i in range(args.warmup):
         step(i, None)
@@ -384,7 +385,7 @@ def run_ours(args):
     if clocks:
         clocks.start()
         time.sleep(0.3)
-    acc = {a: {"ms": 0.0, "edges": 0, "calls": 0} for a in algs}
+    acc = {a: {"ms": 0.0, "edges": 0, "calls": 0, "rates": []} for a in algs}
     launches0 = etg.kernel_launches()
     barrier(world)
     torch.cuda.synchronize()
@@ -407,7 +408,12 @@ def run_ours(args):
     for a in algs:
         ms_a = allreduce([acc[a]["ms"]], tdist.ReduceOp.MAX if world > 1 else None, world)[0]
         e_a = allreduce([float(acc[a]["edges"])], tdist.ReduceOp.SUM if world > 1 else None, world)[0]
-        per_alg[a] = {"gteps": e_a / ms_a / 1e6, "ms_per_call": acc[a]["ms"] / max(1, acc[a]["calls"])}
+        rates = acc[a]["rates"]
+        per_alg[a] = {"gteps": e_a / ms_a / 1e6, "ms_per_call": acc[a]["ms"] / max(1, acc[a]["calls"]),
+                      # per call (one source each): Graph500-style harmonic mean, min, max
+                      "gteps_per_call_hmean": len(rates) / sum(1.0 / r for r in rates) if rates else None,
+                      "gteps_per_call_min": min(rates) if rates else None,
+                      "gteps_per_call_max": max(rates) if rates else None}
     value = tot_edges / max_ms / 1e6
 
     # ---- roofline pass: CUDA events around every expand launch (ETG_PROFILE) ----
