@@ -86,8 +86,9 @@ typedef struct {
                                 deferred; the threshold advances by sssp_delta after every
                                 iteration (and jumps past an empty gap).  Same distances (unique
                                 fixpoint), fewer redundant relaxations.  ETG_SSSP_DELTA_AUTO:
-                                3/8 of the mean edge weight (one O(m) reduction at the first SSSP
-                                call of the handle; 12 for the 1..64 weights of the configs).
+                                6 x mean edge weight / mean out-degree, at least 1 (one O(m)
+                                reduction at the first SSSP call of the handle; 12 / 13 / 6 for
+                                the C2 / C3 / C4 configs).
                                 The step-wise (multi-GPU) API honours it too: the deferred
                                 vertices keep a stale snapshot, identical on every rank. */
 } etg_options;
