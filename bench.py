@@ -56,8 +56,8 @@ def parse_args():
     p.add_argument("--sssp-delta", default="auto",
                    help="SSSP wave schedule: vertices at distance >= a threshold that advances by this much "
                         "every iteration wait (0: the paper's schedule, every improved vertex every iteration; "
-                        "auto: 3/8 of the mean edge weight = 12 for the configs' 1..64 weights, the value "
-                        "measured best on C2), DESIGN.md sec. 5")
+                        "auto: 6 x mean weight / mean out-degree = 12 on C2, 13 on C3, 6 on C4, each near "
+                        "its measured best), DESIGN.md sec. 5")
     p.add_argument("--flags", type=int, default=0, help="extra ETG_* flags (e.g. 2 = NO_UDC)")
     p.add_argument("--sources", type=int, default=16)
     p.add_argument("--no-e2e", action="store_true")
