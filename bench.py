@@ -11,9 +11,14 @@ value = traversed edges / device time, summed over the step's three calls
 nnz of the symmetric CSR for CC).  Inputs are resident in HBM; L2 is flushed
 (256 MiB write) before every traversal call, outside the timed events.
 
-Under torchrun (N > 1) every rank runs its own sources on its own GPU
-(independent problems, no data-path collective): "scaling": "weak", value =
-edges of all ranks / max over ranks of the device time.
+--gpus N > 1 (torchrun, or bench.py relaunches itself under
+torch.distributed.run when WORLD_SIZE is unset): the SAME workload split over
+the N ranks (1-D destination partition) through the library's
+communicator -- every call runs the partitioned loop with the exchange done
+by the library's kernels over peer memory; "scaling": "strong", value = the
+same edges / the per-call device time, max over ranks.  Ranks share a GPU when
+fewer devices than ranks are visible (tests; no speed-up expected there).
+--replicas keeps the older mode: N independent replicas, "scaling": "weak".
 
 --impl reference times the CPU oracle (oracle/, the paper's definitions written
 out plainly) on the host cores, on a bounded sample of the same workload.
@@ -66,15 +71,13 @@ def parse_args():
     p.add_argument("--json-out", default=None)
     p.add_argument("--host-edges", action="store_true",
                    help="NEXT-2: keep col/w in pinned host memory (zero-copy reads by the kernels)")
-    p.add_argument("--partitioned", action="store_true",
-                   help="1-D destination partition of ONE graph over the N ranks (NCCL exchange); "
-                        "default: N independent replicas")
-    p.add_argument("--push", choices=["off", "auto", "sparse", "dense", "p2p"], default="off",
-                   help="with --partitioned: SSSP/CC on a SOURCE partition with the push exchange (NEXT-3: "
-                        "all-to-all of proposals / dense reduce-scatter, auto picks per iteration; p2p: the "
-                        "expand kernel reduces into the owners' label arrays over CUDA-IPC-mapped peer "
-                        "memory); BFS keeps the destination partition (with p2p: owners store their new "
-                        "bitmap words straight into the peers' copies instead of the NCCL all-gather)")
+    p.add_argument("--replicas", action="store_true",
+                   help="N > 1: N independent replicas (own sources per rank, weak scaling) instead of "
+                        "one graph partitioned over the N ranks")
+    p.add_argument("--push", action="store_true",
+                   help="N > 1: SSSP/CC on a SOURCE partition with the fused push exchange (NEXT-3: the "
+                        "expand kernel reduces into the owners' labels over peer memory); BFS keeps the "
+                        "destination partition")
     return p.parse_args()
 
 
@@ -82,16 +85,18 @@ def parse_args():
 # distributed plumbing
 # --------------------------------------------------------------------------- #
 def dist_setup():
+    """Rank / world from the torchrun env.  torch.distributed (gloo) is host
+    plumbing only: the communicator id, barriers around the timed region and
+    the max-over-ranks reduction of a few numbers; no data-path collective."""
     import torch
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    ndev = max(1, torch.cuda.device_count())
+    torch.cuda.set_device(local % ndev)
     if world > 1:
         import torch.distributed as dist
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    elif torch.cuda.is_available():
-        torch.cuda.set_device(0)
+        dist.init_process_group("gloo")
     return rank, world, local
 
 
@@ -106,9 +111,21 @@ def allreduce(vals, op, world):
         return vals
     import torch
     import torch.distributed as dist
-    t = torch.tensor(vals, dtype=torch.float64, device="cuda")
+    t = torch.tensor(vals, dtype=torch.float64)
     dist.all_reduce(t, op=op)
     return t.tolist()
+
+
+def relaunch(args):
+    """--gpus N > 1 without a torchrun environment: run this script under
+    torch.distributed.run with N ranks (127.0.0.1), pass its exit code on."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 # --------------------------------------------------------------------------- #
@@ -486,7 +503,7 @@ def run_ours(args):
                 torch.cuda.synchronize()
                 ev0.record(stream)
                 etg.run_host(alg_id[a], o, c, ww, 0 if a == "cc" else s, hout, scratch, K=args.K,
-                             flags=args.flags, sssp_delta=args.sssp_delta)
+                             flags=args.flags, sssp_delta=args.sssp_delta, symmetric=(a == "cc"))
                 ev1.record(stream)
                 torch.cuda.synchronize()
                 e_ms += ev0.elapsed_time(ev1)
@@ -537,9 +554,11 @@ def run_ours(args):
 
 
 def run_partitioned(args):
-    """One graph split over the N ranks: every rank expands the
-    replicated active set over its destination partition; NCCL all-gather of
-    the owned bitmap words / labels per iteration.  Strong scaling: the same traversals at every N."""
+    """The N=1 workload split over the N ranks: per algorithm
+    one communicator handle per rank (1-D destination partition; --push: SSSP/CC
+    on a source partition), every call the whole partitioned loop inside the
+    library.  Strong scaling: the same traversals, sources and edges at every N."""
+    import numpy as np
     import torch
     import torch.distributed as tdist
     import graphgen as gg
@@ -551,62 +570,97 @@ def run_partitioned(args):
         _build.build()
     barrier(world)
     dev = torch.device("cuda", torch.cuda.current_device())
+    comm = edist.comm_from_group(rank, world, device=dev.index)
     algs = args.algs.split(",")
     alg_id = {"bfs": etg.BFS, "sssp": etg.SSSP, "cc": etg.CC}
-    res = {}
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+    res, e2e_acc = {}, {"ms": 0.0, "edges": 0, "h2d": 0, "d2h": 0}
+    launches = 0
+    clocks = ClockSampler(dev.index) if rank == 0 else None
+    clk_started = False
+    shas = {}
     for a in algs:
         g = gg.make(args.config, device=dev, weights=(a == "sssp"), symmetric=(a == "cc"))
+        if rank == 0:
+            shas[g.name + ("+w" if g.w is not None else "")] = g.sha256()
         deg = g.degrees()
         sources = gg.sample_sources(g, args.sources, 4242)           # the same on every rank
-        group = None
-        if world == 1:
-            import torch.distributed as d0
-            if not d0.is_initialized():
-                if "MASTER_ADDR" in os.environ:          # under torchrun: its env:// rendezvous
-                    d0.init_process_group("nccl", device_id=dev)
-                else:
-                    d0.init_process_group("nccl", init_method="tcp://127.0.0.1:29555", rank=0,
-                                          world_size=1, device_id=dev)
-        push = args.push != "off" and a != "bfs"
-        if push:
-            dg = edist.PushDistGraph(g.off, g.col, g.w, g.n, rank, world, K=args.K, flags=args.flags,
-                                     symmetric=(a == "cc"), device=dev, group=group, mode=args.push)
-        else:
-            dg = edist.DistGraph(g.off, g.col, g.w, g.n, rank, world, K=args.K, flags=args.flags,
-                                 symmetric=(a == "cc"), device=dev, group=group,
-                                 exchange="p2p" if args.push == "p2p" else "collective")
-        lo, hi = dg.bounds[rank], dg.bounds[rank + 1]
+        exchange = "push" if (args.push and a != "bfs") else "dest"
+        dg = edist.DistGraph(g.off, g.col, g.w, g.n, comm, exchange=exchange, K=args.K, flags=args.flags,
+                             symmetric=(a == "cc"), sssp_delta=args.sssp_delta, device=dev)
+        lo, hi = dg.lo, dg.hi
         m_sym = g.m
         del g
         torch.cuda.empty_cache()
-        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        out = torch.empty(max(1, hi - lo), dtype=torch.int32, device=dev)
+        m_reach = {}
+        for s in sources[:min(len(sources), args.warmup + args.steps)]:
+            if a == "cc":
+                m_reach[s] = m_sym
+                continue
+            lab, _ = dg.run(alg_id[a], s, out)         # reached set: the same for BFS and SSSP
+            mine = float(deg[lo:hi][lab[:hi - lo] != -1].sum())
+            m_reach[s] = int(allreduce([mine], tdist.ReduceOp.SUM, world)[0])
+        # warm-up, then the timed calls: per call the library's device time, max over ranks
         ms_tot, edges_tot = 0.0, 0
         for i in range(args.warmup + args.steps):
             s = sources[i % len(sources)]
-            barrier(world)
+            if i == args.warmup:
+                if clocks and not clk_started:
+                    clocks.start()
+                    time.sleep(0.3)
+                    clk_started = True
+                l0 = etg.kernel_launches()
+                barrier(world)
+                torch.cuda.synchronize()
+                if clocks and clocks.t0 is None:
+                    clocks.mark("t0")
+            flush.zero_()
             torch.cuda.synchronize()
-            ev0.record()
-            labels, st = dg.run(alg_id[a], s)
-            ev1.record()
-            torch.cuda.synchronize()
+            _, st = dg.run(alg_id[a], s, out)
             if i >= args.warmup:
-                ms_tot += ev0.elapsed_time(ev1)
-                unreached = etg.INF
-                if a == "cc":
-                    edges_tot += m_sym
-                elif push:      # owned slice only (summed over the ranks below)
-                    edges_tot += int(deg[lo:hi][labels[lo:hi].view(torch.int32) != -1].sum())
-                else:
-                    edges_tot += int(deg[labels.view(torch.int32) != -1].sum())
-        if push or args.push == "p2p":
-            dg.close()
-        ms_max = allreduce([ms_tot], tdist.ReduceOp.MAX, world)[0] if world > 1 else ms_tot
-        if push and a != "cc" and world > 1:
-            edges_tot = int(allreduce([float(edges_tot)], tdist.ReduceOp.SUM, world)[0])
-        res[a] = {"gteps": edges_tot / ms_max / 1e6, "ms_per_call": ms_max / args.steps, "edges": edges_tot,
-                  "ms": ms_max}
+                ms_tot += st.ms
+                edges_tot += m_reach[s]
+        torch.cuda.synchronize()
+        barrier(world)
+        launches += etg.kernel_launches() - l0
+        # e2e: the same calls from pinned HOST buffers -- H2D of this rank's
+        # sub-CSR into the buffers the handle borrows, the call, D2H of the owned slice
+        if not args.no_e2e:
+            dev_bufs = [t for t in dg.graph._keep[:3] if t is not None]
+            host_bufs = [t.cpu().pin_memory() for t in dev_bufs]
+            hout = torch.empty(max(1, hi - lo), dtype=torch.int32).pin_memory()
+            ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            for i in range(args.steps):
+                s = sources[(args.warmup + i) % len(sources)]
+                flush.zero_()
+                barrier(world)
+                torch.cuda.synchronize()
+                ev0.record(stream)
+                for d, h in zip(dev_bufs, host_bufs):
+                    d.copy_(h, non_blocking=True)
+                dg.run(alg_id[a], s, out)
+                hout.copy_(out, non_blocking=True)
+                ev1.record(stream)
+                torch.cuda.synchronize()
+                e_ms = allreduce([ev0.elapsed_time(ev1)], tdist.ReduceOp.MAX, world)[0]
+                e2e_acc["ms"] += e_ms
+                e2e_acc["edges"] += m_reach[s]
+                if i == 0:
+                    e2e_acc["h2d"] += int(allreduce([float(sum(h.numel() * 4 for h in host_bufs))],
+                                                    tdist.ReduceOp.SUM, world)[0])
+                    e2e_acc["d2h"] += 4 * dg.n                 # the owned slices of all ranks
+            del host_bufs, dev_bufs
+        res[a] = {"gteps": edges_tot / ms_tot / 1e6, "ms_per_call": ms_tot / args.steps, "edges": edges_tot,
+                  "ms": ms_tot, "exchange": exchange}
+        dg.close()
         del dg, deg
         torch.cuda.empty_cache()
+    if clocks:
+        clocks.mark("t1")
+    clk = clocks.stop() if clocks else None
+    launches = int(allreduce([float(launches)], tdist.ReduceOp.SUM, world)[0])
     tot_e = sum(v["edges"] for v in res.values())
     tot_ms = sum(v["ms"] for v in res.values())
     if rank == 0:
@@ -616,28 +670,48 @@ def run_partitioned(args):
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
             "config": {"workload": config_desc(args.config) + "; " + "+".join(algs) + " per step",
-                       "parallelism": (f"1-D destination partition over {world} GPU(s), NCCL all-gather exchange of owned slices"
-                                       if args.push == "off" else
-                                       f"SSSP/CC: 1-D source partition over {world} GPU(s), push exchange ({args.push}: "
-                                       f"NCCL all-to-all of proposals or reduce-scatter of labels); BFS: destination partition"),
-                       "K": args.K, "flags": args.flags},
-            "per_alg": {k: {"gteps": v["gteps"], "ms_per_call": v["ms_per_call"]} for k, v in res.items()},
+                       "parallelism": (f"1-D vertex partition over {world} rank(s) "
+                                       f"({'SSSP/CC source partition + fused push exchange, BFS destination' if args.push else 'destination'} "
+                                       "partition), exchange by the library's kernels into the peers' device memory "
+                                       "(CUDA IPC; NVLink between GPUs), host barrier per iteration; "
+                                       f"{torch.cuda.device_count()} visible device(s)"),
+                       "K": args.K, "flags": args.flags, "sources": args.sources,
+                       "sssp_schedule": (f"wave, Delta={args.sssp_delta} (auto from the global sums)"
+                                         if str(args.sssp_delta) != "0" else "paper (Proc. 1)"),
+                       "l2": "flushed (256 MiB write) before every traversal call",
+                       "timing": "per call: the library's CUDA-event device time, max over ranks (etg_stats.ms)",
+                       "sha256": shas},
+            "per_alg": {k: {"gteps": v["gteps"], "ms_per_call": v["ms_per_call"], "exchange": v["exchange"]}
+                        for k, v in res.items()},
+            "roofline": None,
+            "cpu_baseline": None,
+            "e2e": ({"value": e2e_acc["edges"] / e2e_acc["ms"] / 1e6, "unit": UNIT,
+                     "h2d_bytes_per_step": e2e_acc["h2d"], "d2h_bytes_per_step": e2e_acc["d2h"],
+                     "how": "per rank: H2D of its sub-CSR from pinned host memory into the handle's buffers, "
+                            "the call, D2H of the owned label slice; max over ranks"}
+                    if not args.no_e2e and e2e_acc["ms"] > 0 else None),
+            "gpu_launches": launches,
+            "clocks": clk,
         }
-        s = json.dumps(line)
-        print(s, flush=True)
+        out_s = json.dumps(line)
+        print(out_s, flush=True)
         if args.json_out:
             with open(args.json_out, "w") as f:
-                f.write(s + "\n")
-    if torch.distributed.is_initialized():
-        torch.distributed.destroy_process_group()
+                f.write(out_s + "\n")
+    comm.close()
+    if tdist.is_initialized():
+        tdist.destroy_process_group()
     return 0
 
 
 def main():
     args = parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "0"))
     if args.impl == "reference":
         return run_reference(args)
-    if args.partitioned:
+    if args.gpus > 1 and world == 0:
+        return relaunch(args)                  # no torchrun around us: become N ranks
+    if world > 1 and not args.replicas:
         return run_partitioned(args)
     return run_ours(args)
 

@@ -44,13 +44,15 @@ extern "C" {
 #endif
 
 typedef struct etg_graph etg_graph; /* opaque handle */
+typedef struct etg_comm etg_comm;   /* opaque communicator (multi-GPU partitions on one node); NULL = one GPU */
 
 typedef enum {
     ETG_OK = 0,
     ETG_EINVAL = -1,      /* bad argument (NULL pointer, source >= n, K = 0 with UDC, ...) */
     ETG_ENOMEM = -2,      /* workspace too small, or host allocation failed */
     ETG_ECUDA = -3,       /* a CUDA runtime error (detail in etg_last_error) */
-    ETG_ENCCL = -4,       /* reserved for the multi-GPU exchange */
+    ETG_ENCCL = -4,       /* communicator failure: rendezvous, peer mapping, a peer that died or timed out
+                             (ETG_COMM_TIMEOUT_S, default 600 s), ranks that disagree on the graph */
     ETG_ENOTSYM = -5,     /* etg_cc on a handle loaded without ETG_SYMMETRIC */
     ETG_ERANGE = -6,      /* sizes exceed the index types (n > 2^32-2, m >= 2^32 with u32 offsets, ...) */
     ETG_ENOWEIGHTS = -7,  /* etg_sssp / etg_sswp on a handle loaded without weights */
@@ -61,8 +63,8 @@ enum {
     ETG_SYMMETRIC = 1u << 0,   /* caller asserts the CSR is symmetric (required by etg_cc) */
     ETG_NO_UDC = 1u << 1,      /* ablation: one work item per active vertex (K = infinity) */
     ETG_NO_SMP = 1u << 2,      /* ablation ("w/o SMP", Sec. VI-C): no look-ahead fetch of the
-                                  next tile's neighbour segments (default: TMA bulk prefetch
-                                  into L2) */
+                                  next batch's neighbour segments (default: register look-ahead,
+                                  BFS) */
     ETG_OFFSETS_U64 = 1u << 3, /* d_row_offsets holds uint64 (needed when m >= 2^32) */
     ETG_VALIDATE = 1u << 4,    /* etg_load_csr runs an O(n+m) device check of the CSR */
     ETG_HOST_LOOP = 1u << 5,   /* drive iterations from the host (count read back each
@@ -71,10 +73,15 @@ enum {
                                   expand launch on the handle's stream fill scan_ms/expand_ms */
     ETG_SMP_SHARED = 1u << 7,  /* SMP as literally described (L199): TMA bulk copies of the next
                                   tile's segments into per-warp shared-memory stages (K <= 32) */
-    ETG_HOST_EDGES = 1u << 8   /* host-resident edge mode (NEXT-2; Sec. IV-B): d_col_idx
+    ETG_HOST_EDGES = 1u << 8,  /* host-resident edge mode (NEXT-2; Sec. IV-B): d_col_idx
                                   and d_weights point to pinned, device-mapped HOST memory (UVA
                                   zero-copy); each iteration reads only the active vertices' edges
                                   over the host link.  Offsets and workspace stay in HBM. */
+    ETG_PUSH = 1u << 9         /* communicator handles only: the CSR is the rank's SOURCE partition
+                                  (rows v_lo..v_hi-1 keep their out-edges, the others are empty;
+                                  global ids) and the expand kernel reduces every relaxation of a
+                                  foreign vertex into its owner's labels over peer memory (SURVEY
+                                  8(f) NEXT-3).  SSSP/CC/SSWP; etg_bfs returns ETG_EINVAL. */
 };
 
 typedef struct {
@@ -115,14 +122,41 @@ size_t etg_workspace_bytes(uint64_t n, uint64_t m, const etg_options *opt);
 
 /* Create a handle over a caller-owned device CSR (Proc. 1 "Load data", L207;
  * the CSR is used unmodified, L113).  d_weights may be NULL (then SSSP/SSWP
- * return ETG_ENOWEIGHTS).  stream is a cudaStream_t (void* here). */
+ * return ETG_ENOWEIGHTS).  stream is a cudaStream_t (void* here).
+ *
+ * comm == NULL: one GPU; v_lo / v_hi are ignored (the handle owns [0, n)).
+ * comm != NULL (collective: every rank of the communicator calls it, in any
+ * order, each with its own partition): the 1-D vertex partition of SURVEY
+ * 8(e) -- rank r owns [v_lo, v_hi); the ranges must tile [0, n) in rank order
+ * with inner bounds multiples of 32 (one bitmap word, one owner).  n is the
+ * GLOBAL vertex count and m the number of edges of this rank's sub-CSR:
+ *   default (destination partition): rows = all n sources, only the edges
+ *     whose destination lies in [v_lo, v_hi), global ids;
+ *   ETG_PUSH (source partition): rows v_lo..v_hi-1 keep all their out-edges,
+ *     every other row is empty.
+ * The call exchanges the workspaces' CUDA-IPC handles through the
+ * communicator and maps every peer's workspace into this process, so each
+ * traversal's per-iteration exchange is done by the library's kernels writing
+ * into the peers' device memory (NVLink / NVSwitch between GPUs).  Errors:
+ * ETG_EINVAL (range outside [0, n], ETG_PUSH without comm), ETG_ENCCL (ranges
+ * that do not tile [0, n), ranks that disagree on n or ETG_PUSH, a peer that
+ * cannot be mapped or does not arrive). */
 etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m,
                         const void *d_row_offsets, const uint32_t *d_col_idx,
                         const uint32_t *d_weights, void *d_workspace,
-                        size_t workspace_bytes, void *stream, const etg_options *opt);
+                        size_t workspace_bytes, void *stream, const etg_options *opt,
+                        const etg_comm *comm, uint32_t v_lo, uint32_t v_hi);
 
 /* BFS (Proc. 1 Kernel BFS, L207): d_depth[v] = hop distance from source, INF if
- * unreachable. */
+ * unreachable.
+ * On a communicator handle (all four traversals): collective -- every rank
+ * calls it with the same source; the whole partitioned Proc. 1 loop runs
+ * inside the call (per iteration: expand, exchange over peer memory, host
+ * barrier, scan, barrier with the termination count) and the output array
+ * receives the OWNED slice only: v_hi - v_lo entries, d_out[i] = label of
+ * vertex v_lo + i.  Statistics are summed over the ranks; st->ms is the
+ * maximum over the ranks of the call's device time (st->reserved: this
+ * rank's own). */
 etg_status etg_bfs(etg_graph *g, uint32_t source, uint32_t *d_depth, etg_stats *st_or_null);
 
 /* SSSP (L62, L78): d_dist[v] = saturating shortest-path distance (CAP), INF if
@@ -164,20 +198,17 @@ etg_status etg_debug_expand_replay(etg_graph *g, int alg, uint32_t source, uint3
                                    uint32_t tune, int reps, uint32_t *d_label, uint32_t *d_saved,
                                    float *ms, uint64_t *edges, uint32_t *n_active);
 
-/* ---- Step-wise driving (1-D vertex-range partitions over several GPUs, Sec.
- * "Multi-GPU" of DESIGN.md).  A partition's handle is loaded with the
- * rank's destination-partitioned CSR: all n source rows, only the edges whose
- * destination lies in the rank's owned range, global vertex ids.  Labels and
- * the active-set bitmap are full-size (n) on every rank.  Protocol:
- *   etg_step_begin -> while (n_active) { etg_step_expand; exchange;
- *   etg_step_scan } -> etg_step_end,
- * where "exchange" makes every rank's bitmap (etg_bitmap_layout: nwords uint32
- * words at offset_bytes into the workspace) the OR of all ranks' bitmaps and,
- * for SSSP/CC/SSWP, every rank's labels the min (SSWP: max) over ranks.
- * n_active is the number of vertices activated (bitmap bits consumed by the
- * scan); it is identical on every rank after an exchange, so all ranks leave
- * the loop together (a rank whose compacted set is empty expands nothing).
- * etg_step_begin already runs the first scan (the initial active set). */
+/* ---- Step-wise driving of one handle (per-iteration tracing and tuning;
+ * the communicator loop is built from the same steps).  Protocol:
+ *   etg_step_begin -> while (n_active) { etg_step_expand; etg_step_scan } ->
+ *   etg_step_end.
+ * etg_step_begin runs A1 and the first scan (the initial active set);
+ * n_active is the number of vertices the scan activated (bitmap bits
+ * consumed).  The Proc. 1 loop is identical to etg_bfs/... except that the
+ * host reads n_active back every iteration.  etg_bitmap_layout: the active-set
+ * bitmap Q is nwords uint32 words at offset_bytes into the workspace.
+ * ETG_EINVAL: NULL arguments, alg outside 0..3, source >= n, a step without
+ * etg_step_begin, SSSP on a handle loaded with ETG_SSSP_DELTA_AUTO. */
 etg_status etg_step_begin(etg_graph *g, int alg, uint32_t source, uint32_t *d_label,
                           uint32_t *n_active);
 etg_status etg_step_expand(etg_graph *g);
@@ -185,70 +216,10 @@ etg_status etg_step_scan(etg_graph *g, uint32_t *n_active);
 etg_status etg_step_end(etg_graph *g, etg_stats *st_or_null);
 etg_status etg_bitmap_layout(etg_graph *g, size_t *offset_bytes, uint32_t *nwords);
 
-/* ---- NEXT-3 push exchange (the all-to-all option of the
- * north star's item 4).  SOURCE partition: a rank's handle is loaded with the
- * out-edges of its owned range [bounds[rank], bounds[rank+1]) only (other
- * rows empty, global ids), so its relaxations (Proc. 1 L207) land on any
- * vertex.  SSSP/CC/SSWP only (BFS keeps the destination partition), no
- * near-far.  After etg_step_expand, every vertex v this rank does NOT own whose
- * label moved (label != snapshot) carries a proposal for v's owner:
- *   etg_push_count: d_counts[q] = number of proposals for owner q
- *     (device, P entries of uint64, overwritten; d_counts[rank] = 0).
- *   etg_push_pack: appends (v, label[v]) uint32 pairs to d_pairs, owner q's
- *     proposals at pair index d_cursor[q] onwards (device, P uint64 entries,
- *     typically the exclusive scan of the counts; advanced by the call; order
- *     inside a segment unspecified), and marks them sent (snapshot = label).
- *   etg_push_apply: label[v] = min(label[v], val) (SSWP: max) for `count`
- *     received pairs (device memory, 2 * count uint32).
- * Then etg_step_scan activates the owned vertices whose label moved.  The
- * caller moves the pairs (all-to-all) or, when that is more bytes, reduces the
- * full label arrays (MIN; SSWP MAX) onto each owner's range instead, and
- * stops when the compacted active sets of all ranks are empty
- * (etg_debug_counters out[1]).  d_bounds: P + 1 uint32 in device memory,
- * bounds[0] = 0, bounds[P] = n, inner bounds multiples of 32.  Errors:
- * ETG_EINVAL on NULL pointers, P > 64, rank >= P, or no SSSP/CC/SSWP step run. */
-etg_status etg_push_count(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *d_bounds,
-                          unsigned long long *d_counts);
-etg_status etg_push_pack(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *d_bounds,
-                         unsigned long long *d_cursor, uint32_t *d_pairs);
-etg_status etg_push_apply(etg_graph *g, const uint32_t *d_pairs, uint64_t count);
+/* The SSSP wave width Delta the handle uses (etg_options.sssp_delta; auto is
+ * resolved here if no SSSP ran yet -- collective on a communicator handle). */
+etg_status etg_sssp_delta(etg_graph *g, uint32_t *delta);
 
-/* Fused push exchange over peer memory (the north star's "one kernel that does
- * both over peer memory"; replaces count/pack/all-to-all/apply).  After this
- * call, every etg_step_expand of the handle (SSSP/CC/SSWP) applies each
- * improving relaxation of a vertex u owned by rank q != rank (h_bounds[q] <=
- * u < h_bounds[q+1]) twice: to its own label array (the proposal cache that
- * filters repeats) and, as a system-scope red.min (SSWP: red.max), to
- * h_peer_labels[q][u] -- rank q's label array, mapped into this process
- * (etg_ipc_open of the peer's etg_ipc_handle on another GPU over NVLink, or a
- * plain device pointer for partitions sharing a GPU).  h_peer_labels[rank] is
- * unused.  The caller makes every rank's expand complete (stream sync + host
- * barrier) before any rank's etg_step_scan, which then activates the owned
- * vertices whose label moved.  h_bounds: host, P + 1 entries, 0 .. n.
- * P = 0 turns it off.  ETG_EINVAL: P > 8, rank >= P, bad bounds, NULL
- * pointers, or a handle without the warp expand kernel. */
-etg_status etg_push_peers(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *h_bounds,
-                          uint32_t *const *h_peer_labels);
-/* Fused destination-partition exchange (replaces the exchange of the
- * step-wise protocol above for destination partitions): register every
- * rank's bitmap Q (etg_bitmap_layout) and label array, mapped into this
- * process, and the partition bounds (host, P + 1 entries, inner bounds
- * multiples of 32).  etg_step_publish, called after etg_step_expand, then
- * stores what changed in this rank's owned range straight into every peer's
- * copy: BFS -- the non-zero bitmap words (only the owner marks its vertices,
- * so a plain store is the union); SSSP/CC/SSWP -- the labels that moved
- * (label != snapshot).  The caller waits for every rank's publish (stream
- * sync + host barrier) before the scans.  P = 0 turns it off; ETG_EINVAL on
- * bad arguments, or publish without peers / outside a step-wise run. */
-etg_status etg_dest_peers(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *h_bounds,
-                          uint32_t *const *h_peer_Q, uint32_t *const *h_peer_labels);
-etg_status etg_step_publish(etg_graph *g);
-/* CUDA IPC for the peer label arrays: the handle (64 bytes) of the allocation
- * holding d_ptr and d_ptr's byte offset in it; open maps a peer's handle into
- * this process (base address; add the offset), close unmaps it. */
-etg_status etg_ipc_handle(const void *d_ptr, uint8_t *out_handle, uint64_t *out_offset);
-etg_status etg_ipc_open(const uint8_t *handle, void **out_base);
-etg_status etg_ipc_close(void *base);
 /* Tracing (step-wise runs): the device counters as of the last etg_step_* call
  * that synchronised (begin/scan/end): out[0] depth, [1] compacted active-set
  * size |F| (Proc. 1 actSet, L207), [2] shadow vertices of F (Def. 3),
@@ -275,6 +246,24 @@ etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_row_offse
                         uint32_t source, uint32_t *h_labels, void *d_scratch,
                         size_t scratch_bytes, void *stream, const etg_options *opt,
                         etg_stats *st_or_null);
+
+/* ---- Communicator (one process -- or thread -- per partition on
+ * ONE node).  Rank 0 calls etg_comm_unique_id and hands the 128 bytes to the
+ * other ranks by any means (the binding uses torch.distributed); every rank
+ * then calls etg_comm_init with its rank, the world size (1..8) and the CUDA
+ * device it drives (-1: the calling thread's current device).  The
+ * communicator is the control plane only -- a POSIX shared-memory segment
+ * with one slot per rank (workspace IPC handles, owned ranges, termination
+ * counts) and a host barrier; the data plane is the library's kernels.
+ * etg_comm_init blocks until all `world` ranks have joined.  Errors:
+ * ETG_EINVAL (rank >= world, world outside 1..8, not a unique id, rank
+ * taken twice), ETG_ENCCL (shared memory unavailable, timeout, a peer died).
+ * etg_comm_barrier: a host barrier over the ranks (plumbing and tests).
+ * etg_comm_free after every handle loaded with it has been freed. */
+etg_status etg_comm_unique_id(uint8_t *id /* 128 bytes */);
+etg_status etg_comm_init(etg_comm **out, int rank, int world, const uint8_t *id, int device);
+etg_status etg_comm_barrier(const etg_comm *comm);
+void etg_comm_free(etg_comm *comm);
 
 const char *etg_status_str(etg_status s);
 const char *etg_last_error(void);

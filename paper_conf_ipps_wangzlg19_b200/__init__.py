@@ -22,14 +22,14 @@ import torch
 
 __all__ = [
     "EtgError", "Stats", "Graph", "load_csr", "csr_to_device", "to_u32_numpy",
-    "run_host", "host_scratch_bytes", "kernel_launches", "lib",
+    "run_host", "host_scratch_bytes", "kernel_launches", "lib", "Comm",
     "SYMMETRIC", "NO_UDC", "NO_SMP", "OFFSETS_U64", "VALIDATE", "HOST_LOOP", "PROFILE", "SMP_SHARED",
-    "HOST_EDGES",
+    "HOST_EDGES", "PUSH",
     "INF", "CAP", "BFS", "SSSP", "CC", "SSWP",
 ]
 
-SYMMETRIC, NO_UDC, NO_SMP, OFFSETS_U64, VALIDATE, HOST_LOOP, PROFILE, SMP_SHARED, HOST_EDGES = (
-    1, 2, 4, 8, 16, 32, 64, 128, 256)
+SYMMETRIC, NO_UDC, NO_SMP, OFFSETS_U64, VALIDATE, HOST_LOOP, PROFILE, SMP_SHARED, HOST_EDGES, PUSH = (
+    1, 2, 4, 8, 16, 32, 64, 128, 256, 512)
 INF, CAP = 0xFFFFFFFF, 0xFFFFFFFE
 BFS, SSSP, CC, SSWP = 0, 1, 2, 3
 
@@ -72,7 +72,11 @@ def lib():
         st = ctypes.c_int
         sig = {
             "etg_workspace_bytes": (sz, [u64, u64, p]),
-            "etg_load_csr": (st, [ctypes.POINTER(p), u64, u64, p, p, p, p, sz, p, p]),
+            "etg_load_csr": (st, [ctypes.POINTER(p), u64, u64, p, p, p, p, sz, p, p, p, u32, u32]),
+            "etg_comm_unique_id": (st, [p]),
+            "etg_comm_init": (st, [ctypes.POINTER(p), ctypes.c_int, ctypes.c_int, p, ctypes.c_int]),
+            "etg_comm_barrier": (st, [p]),
+            "etg_comm_free": (None, [p]),
             "etg_bfs": (st, [p, u32, p, p]),
             "etg_sssp": (st, [p, u32, p, p]),
             "etg_cc": (st, [p, p, p]),
@@ -91,15 +95,7 @@ def lib():
             "etg_step_scan": (st, [p, ctypes.POINTER(u32)]),
             "etg_step_end": (st, [p, p]),
             "etg_bitmap_layout": (st, [p, ctypes.POINTER(sz), ctypes.POINTER(u32)]),
-            "etg_push_count": (st, [p, u32, u32, p, p]),
-            "etg_push_pack": (st, [p, u32, u32, p, p, p]),
-            "etg_push_apply": (st, [p, p, u64]),
-            "etg_push_peers": (st, [p, u32, u32, p, p]),
-            "etg_ipc_handle": (st, [p, p, ctypes.POINTER(u64)]),
-            "etg_ipc_open": (st, [p, ctypes.POINTER(p)]),
-            "etg_ipc_close": (st, [p]),
-            "etg_dest_peers": (st, [p, u32, u32, p, p, p]),
-            "etg_step_publish": (st, [p]),
+            "etg_sssp_delta": (st, [p, ctypes.POINTER(u32)]),
             "etg_debug_expand_replay": (st, [p, ctypes.c_int, u32, u32, u32, ctypes.c_int, p, p,
                                              ctypes.POINTER(ctypes.c_float), ctypes.POINTER(u64),
                                              ctypes.POINTER(u32)]),
@@ -116,7 +112,8 @@ SSSP_DELTA_AUTO = 0xFFFFFFFF
 
 
 def _delta(d) -> int:
-    """sssp_delta: an int (0 = the paper's schedule) or "auto" (3/8 of the mean weight)."""
+    """sssp_delta: an int (0 = the paper's schedule) or "auto" (6 x mean edge
+    weight / mean out-degree, at least 1: 12 / 13 / 6 on C2 / C3 / C4)."""
     return SSSP_DELTA_AUTO if d == "auto" else int(d)
 
 
@@ -170,12 +167,52 @@ def csr_to_device(off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor
     return off_d, col_d, w_d, flags
 
 
+class Comm:
+    """A communicator over the ranks of one node (etg_comm_init).  Rank 0 makes
+    the id with :meth:`unique_id`; the caller hands it to the other ranks
+    (e.g. torch.distributed.broadcast_object_list -- bootstrap only)."""
+
+    def __init__(self, rank: int, world: int, uid: bytes, device: int = -1):
+        if len(uid) != 128:
+            raise EtgError("unique id must be 128 bytes")
+        h = ctypes.c_void_p()
+        _check(lib().etg_comm_init(ctypes.byref(h), rank, world, (ctypes.c_uint8 * 128)(*uid), device),
+               "etg_comm_init")
+        self._h = h
+        self.rank, self.world, self.device = rank, world, device
+
+    @staticmethod
+    def unique_id() -> bytes:
+        buf = (ctypes.c_uint8 * 128)()
+        _check(lib().etg_comm_unique_id(buf), "etg_comm_unique_id")
+        return bytes(buf)
+
+    def barrier(self) -> None:
+        _check(lib().etg_comm_barrier(self._h), "etg_comm_barrier")
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().etg_comm_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 class Graph:
-    """A handle over a device CSR (etg_load_csr).  Keeps its tensors alive."""
+    """A handle over a device CSR (etg_load_csr).  Keeps its tensors alive.
+
+    With ``comm`` (a :class:`Comm`): this rank's partition of a graph of ``n``
+    vertices owning [v_lo, v_hi) (see include/etg.h); construction is
+    collective, every traversal is collective and returns the owned slice."""
 
     def __init__(self, off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor] = None, *,
                  n: Optional[int] = None, K: int = 32, flags: int = 0, symmetric: bool = False,
-                 validate: bool = False, stream=None, sssp_delta: int = 0):
+                 validate: bool = False, stream=None, sssp_delta: int = 0, comm: Optional[Comm] = None,
+                 v_lo: int = 0, v_hi: Optional[int] = None):
         if not torch.cuda.is_available():
             raise EtgError("no CUDA device: etg has no CPU fallback")
         if off.dtype == torch.int64:
@@ -203,8 +240,11 @@ class Graph:
         self.device = off.device
         if not off.is_cuda:
             raise EtgError("row offsets must live on the device")
-        self._keep = (off, col, w)
+        self._keep = (off, col, w, comm)
         self._stream = stream
+        self.comm = comm
+        self.v_lo = v_lo if comm is not None else 0
+        self.v_hi = (self.n if v_hi is None else v_hi) if comm is not None else self.n
         self._opt = Options(K, flags, _delta(sssp_delta))
         L = lib()
         nbytes = L.etg_workspace_bytes(self.n, self.m, ctypes.byref(self._opt))
@@ -212,16 +252,18 @@ class Graph:
         h = ctypes.c_void_p()
         rc = L.etg_load_csr(ctypes.byref(h), self.n, self.m, _ptr(off), _ptr(col), _ptr(w),
                             _ptr(self.workspace), nbytes, _stream_ptr(stream),
-                            ctypes.byref(self._opt))
+                            ctypes.byref(self._opt), None if comm is None else comm._h,
+                            self.v_lo, self.v_hi)
         _check(rc, "etg_load_csr")
         self._h = h
 
     # -- traversals --------------------------------------------------------- #
     def _out(self, out):
+        k = self.v_hi - self.v_lo            # n, or the owned slice of a partition
         if out is None:
-            out = torch.empty(self.n, dtype=torch.int32, device=self.device)
-        if out.dtype != torch.int32 or out.numel() < self.n or not out.is_contiguous():
-            raise EtgError("out must be a contiguous int32 tensor of n entries")
+            out = torch.empty(max(k, 1), dtype=torch.int32, device=self.device)
+        if out.dtype != torch.int32 or out.numel() < k or not out.is_contiguous():
+            raise EtgError(f"out must be a contiguous int32 tensor of {k} entries")
         return out
 
     def bfs(self, source: int, out: Optional[torch.Tensor] = None):
@@ -256,6 +298,12 @@ class Graph:
         if alg == CC:
             return self.cc(out)
         return self.sswp(source, out)
+
+    def sssp_delta(self) -> int:
+        """The SSSP wave width Delta of this handle (auto resolved on first use)."""
+        d = ctypes.c_uint32()
+        _check(lib().etg_sssp_delta(self._h, ctypes.byref(d)), "etg_sssp_delta")
+        return int(d.value)
 
     def reach_stats(self, labels: torch.Tensor, unreached: int = INF) -> Stats:
         st = Stats()
@@ -318,14 +366,16 @@ def host_scratch_bytes(n: int, m: int, has_weights: bool, K: int = 32, flags: in
 
 def run_host(alg: int, off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor],
              source: int, labels_out: torch.Tensor, scratch: torch.Tensor, *, K: int = 32,
-             flags: int = 0, stream=None, sssp_delta: int = 0) -> Stats:
-    """End-to-end call on HOST tensors (pinned recommended): H2D, traverse, D2H."""
+             flags: int = 0, stream=None, sssp_delta: int = 0, symmetric: bool = False) -> Stats:
+    """End-to-end call on HOST tensors (pinned recommended): H2D, traverse, D2H.
+    CC needs ``symmetric=True`` (the caller asserts the CSR is symmetric, as
+    with :class:`Graph`); without it the library returns ETG_ENOTSYM."""
     for t in (off, col, w, labels_out):
         if t is not None and t.is_cuda:
             raise EtgError("run_host takes host tensors")
     if off.dtype == torch.int64:
         flags |= OFFSETS_U64
-    if alg == CC:
+    if symmetric:
         flags |= SYMMETRIC
     n = int(off.shape[0] - 1)
     m = int(col.shape[0])

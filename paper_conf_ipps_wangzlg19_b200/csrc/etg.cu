@@ -20,6 +20,7 @@
 #include <string>
 
 #include "../../include/etg.h"
+#include "etg_comm.h"
 #include "etg_kernels.cuh"
 
 using namespace etg;
@@ -104,7 +105,7 @@ Params derive(const etg_options *opt, uint32_t tune) {
 }
 
 struct Layout {
-    size_t Q, V, snap, F, B, D, S, Lx, tile_first, recE, recS, ctl, total;
+    size_t Q, Lfull, V, snap, F, B, D, S, Lx, tile_first, recE, recS, ctl, total;
     uint32_t nwords;
 };
 
@@ -123,6 +124,7 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
     const uint64_t tile_words = kScanV / 32;
     L.nwords = (uint32_t)((words + tile_words - 1) / tile_words * tile_words);
     L.Q = take(4ull * L.nwords);
+    L.Lfull = take(4 * (n + 1));   // communicator handles: the full-size label array (peers write into it)
     L.V = take(4ull * L.nwords);
     L.snap = take(4 * (n + 1));
     L.F = take(4 * (n + 1));
@@ -139,6 +141,10 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
 }
 
 }  // namespace
+
+struct etg_comm {
+    etg::Comm c;
+};
 
 struct etg_graph {
     uint64_t n = 0, m = 0;
@@ -160,15 +166,20 @@ struct etg_graph {
     cudaEvent_t pev[3] = {nullptr, nullptr, nullptr};   // ETG_PROFILE: scan / expand brackets
     int step_alg = -1;                    // algorithm of the step-wise (distributed) run
     uint32_t *step_label = nullptr;       // its label array
-    uint32_t npeer = 0, peer_rank = 0;    // fused push exchange (etg_push_peers)
+    uint32_t npeer = 0, peer_rank = 0;    // ETG_PUSH communicator handles: the fused push exchange
     uint32_t peer_bounds[kMaxPeer + 1] = {};
     uint32_t *peer_label[kMaxPeer] = {};
-    uint32_t dpeer = 0, dpeer_rank = 0;   // fused destination-partition exchange (etg_dest_peers)
+    uint32_t dpeer = 0, dpeer_rank = 0;   // destination-partition communicator handles: publish targets
     uint32_t dpeer_lo = 0, dpeer_hi = 0;
     uint32_t *dpeer_Q[kMaxPeer] = {};
     uint32_t *dpeer_label[kMaxPeer] = {};
     uint64_t step_launches = 0;
     uint64_t step_acts = 0;               // activations counted so far (cumulative)
+    bool delta_auto = false;              // sssp_delta was ETG_SSSP_DELTA_AUTO at load (sticky)
+    etg::Comm *comm = nullptr;            // communicator (borrowed), NULL = single partition
+    bool push = false;                    // ETG_PUSH: source partition + fused push exchange
+    uint32_t v_lo = 0, v_hi = 0;          // owned vertex range
+    void *ipc_base[kMaxPeer] = {};        // peer workspaces mapped with cudaIpcOpenMemHandle
     cudaGraphExec_t exec[4] = {nullptr, nullptr, nullptr, nullptr};
     int grid_loop[4] = {0, 0, 0, 0};      // loop_kernel grid per algorithm (resident CTAs x SMs)
     cudaGraph_t graph[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -555,10 +566,36 @@ etg_status step_expand_impl(etg_graph *g) {
     return ETG_OK;
 }
 
-// ETG_SSSP_DELTA_AUTO: Delta = 6 x mean edge weight / mean out-degree (>= 1), resolved once per handle.
+// ---- communicator plumbing (etg_comm_*; host control plane in etg_comm.h) ----
+etg_status comm_fail(int rc, const char *what) {
+    return fail(ETG_ENCCL, std::string(what) + (rc == -2 ? ": a peer process died" : ": timed out waiting for the peers"));
+}
+
+#define ETG_BAR(c, what)                                   \
+    do {                                                   \
+        const int brc_ = etg::comm_barrier(c);             \
+        if (brc_) return comm_fail(brc_, what);            \
+    } while (0)
+
+// All-gather of k <= kCommVals 64-bit values at slot positions [at, at + k):
+// write, barrier, read.  No trailing barrier: every caller uses positions that
+// are rewritten only after at least one more barrier.
+etg_status comm_gather(const etg::Comm &c, int at, const uint64_t *mine, int k,
+                       uint64_t (*out)[etg::kCommVals]) {
+    for (int i = 0; i < k; ++i) c.sh->slot[c.rank].val[at + i] = mine[i];
+    ETG_BAR(c, "all-gather");
+    for (int q = 0; q < c.world; ++q)
+        for (int i = 0; i < k; ++i) out[q][at + i] = c.sh->slot[q].val[at + i];
+    return ETG_OK;
+}
+
+// ETG_SSSP_DELTA_AUTO: Delta = 6 x mean edge weight / mean out-degree (>= 1),
+// resolved once per handle; on a communicator handle from the GLOBAL sums (all
+// ranks then run the same schedule as the single-GPU call).
 etg_status resolve_delta(etg_graph *g) {
     if (g->p.nf_delta != ETG_SSSP_DELTA_AUTO) return ETG_OK;
     uint32_t delta = 1;
+    unsigned long long wsum = 0;
     if (g->m && g->w) {
         ETG_CU(cudaMemsetAsync(&g->ctl->reached_e, 0, sizeof(unsigned long long), g->stream));
         weight_sum_kernel<<<g->grid_init, kBlock, 0, g->stream>>>(g->w, g->m, g->ctl);
@@ -566,14 +603,131 @@ etg_status resolve_delta(etg_graph *g) {
         ETG_CU(cudaMemcpyAsync(&g->h_ctl->reached_e, &g->ctl->reached_e, sizeof(unsigned long long),
                                cudaMemcpyDeviceToHost, g->stream));
         ETG_CU(cudaStreamSynchronize(g->stream));
+        wsum = g->h_ctl->reached_e;
+    }
+    uint64_t m = g->m;
+    if (g->comm && g->comm->world > 1) {
+        uint64_t mine[2] = {wsum, g->m}, all[etg::kCommMaxRanks][etg::kCommVals];
+        etg_status rc = comm_gather(*g->comm, 8, mine, 2, all);   // positions 8, 9: only used here
+        if (rc != ETG_OK) return rc;
+        wsum = 0;
+        m = 0;
+        for (int q = 0; q < g->comm->world; ++q) {
+            wsum += all[q][8];
+            m += all[q][9];
+        }
+    }
+    if (m && wsum) {
         // 6 x mean weight / mean out-degree: C2 (deg 16) 12, C3 (14.4) 13,
         // C4 (35.3) 6 -- each within a few % of its measured best Delta
-        const double mean_w = (double)g->h_ctl->reached_e / (double)g->m;
-        const double mean_deg = (double)g->m / (double)(g->n ? g->n : 1);
+        const double mean_w = (double)wsum / (double)m;
+        const double mean_deg = (double)m / (double)(g->n ? g->n : 1);
         const double d = 6.0 * mean_w / mean_deg + 0.5;
         delta = d < 1.0 ? 1u : (d > 2147483647.0 ? 0x7FFFFFFFu : (uint32_t)d);
     }
     g->p.nf_delta = delta;
+    return ETG_OK;
+}
+
+etg_status publish_impl(etg_graph *g);
+
+// The whole partitioned traversal of one rank (Proc. 1 L207 on a
+// 1-D vertex partition).  Destination partition (default): every rank expands
+// the replicated active set over its sub-CSR (edges INTO its range), relaxes
+// owned vertices only, then publishes what changed in its range straight into
+// every peer's copy (publish_kernel over peer memory); push partition
+// (ETG_PUSH): every rank expands its own vertices and the expand kernel itself
+// reduces each relaxation of a foreign vertex into the owner's labels.
+// Per iteration: expand [-> publish] -> stream sync -> barrier -> scan ->
+// barrier with the termination count.  The count is identical on every rank
+// in the destination partition (checked); the push partition stops when no
+// rank has work left.
+template <class OffT>
+etg_status comm_run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *out, etg_stats *st) {
+    const etg::Comm &c = *g->comm;
+    cudaStream_t s = g->stream;
+    uint32_t *lab = reinterpret_cast<uint32_t *>(g->ws + g->L.Lfull);
+    const bool multi = c.world > 1;
+    uint64_t all[etg::kCommMaxRanks][etg::kCommVals];
+    ETG_CU(cudaEventRecord(g->ev0, s));
+    uint32_t nact = 0;
+    etg_status rc = step_begin_impl<OffT>(g, alg, source, lab, &nact, 0);
+    if (rc != ETG_OK) return rc;
+    ETG_BAR(c, "init");                  // every copy initialised before anyone writes into it
+    auto live_count = [&](uint64_t &live) -> etg_status {
+        // push: any rank with work (compacted vertices or deferred far ones);
+        // destination: the activation count, identical on every rank
+        uint64_t mine = g->push ? (uint64_t)g->h_ctl->more : (uint64_t)nact;
+        if (!multi) {
+            live = mine;
+            return ETG_OK;
+        }
+        etg_status r = comm_gather(c, 0, &mine, 1, all);
+        if (r != ETG_OK) return r;
+        live = 0;
+        for (int q = 0; q < c.world; ++q) {
+            if (!g->push && all[q][0] != mine)
+                return fail(ETG_ENCCL, "ranks disagree on the active-set size (not the same graph or arguments?)");
+            live += all[q][0];
+        }
+        return ETG_OK;
+    };
+    uint64_t live = 0;
+    rc = live_count(live);
+    if (rc != ETG_OK) return rc;
+    while (live) {
+        rc = step_expand_impl<OffT>(g);
+        if (rc != ETG_OK) return rc;
+        if (!g->push && multi) {
+            rc = publish_impl(g);
+            if (rc != ETG_OK) return rc;
+        }
+        if (multi) {
+            ETG_CU(cudaStreamSynchronize(s));
+            ETG_BAR(c, "exchange");      // every rank's writes into this rank's copy have landed
+        }
+        rc = step_scan_impl<OffT>(g, &nact);
+        if (rc != ETG_OK) return rc;
+        rc = live_count(live);           // also: nobody writes iteration k+1 into a copy still being scanned
+        if (rc != ETG_OK) return rc;
+    }
+    ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    if (g->v_hi > g->v_lo)
+        ETG_CU(cudaMemcpyAsync(out, lab + g->v_lo, 4ull * (g->v_hi - g->v_lo), cudaMemcpyDeviceToDevice, s));
+    ETG_CU(cudaEventRecord(g->ev1, s));
+    ETG_CU(cudaStreamSynchronize(s));
+    ETG_CU(cudaGetLastError());
+    g_launches += g->step_launches + 1;
+    g->step_alg = -1;
+    float ms = 0.f;
+    ETG_CU(cudaEventElapsedTime(&ms, g->ev0, g->ev1));
+    const Ctl &h = *g->h_ctl;
+    uint64_t mine[5] = {h.edges, h.shadows, h.frontier, h.activations, 0};
+    memcpy(&mine[4], &ms, sizeof(float));
+    uint64_t tot[5] = {mine[0], mine[1], mine[2], mine[3], 0};
+    float ms_max = ms;
+    if (multi) {
+        rc = comm_gather(c, 1, mine, 5, all);
+        if (rc != ETG_OK) return rc;
+        for (int i = 0; i < 4; ++i) tot[i] = 0;
+        for (int q = 0; q < c.world; ++q) {
+            for (int i = 0; i < 4; ++i) tot[i] += all[q][1 + i];
+            float mq = 0.f;
+            memcpy(&mq, &all[q][5], sizeof(float));
+            ms_max = std::max(ms_max, mq);
+        }
+        if (!g->push) tot[3] = h.activations;   // replicated active set: the same on every rank
+    }
+    if (st) {
+        memset(st, 0, sizeof(*st));
+        st->iterations = h.iterations;
+        st->edges_processed = tot[0];
+        st->shadows = tot[1];
+        st->frontier_total = tot[2];
+        st->activations = tot[3];
+        st->ms = ms_max;                 // max over ranks
+        st->reserved = ms;               // this rank's own device time
+    }
     return ETG_OK;
 }
 
@@ -587,6 +741,12 @@ etg_status run(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stat
     }
     if (alg == ALG_CC && !(g->flags & ETG_SYMMETRIC)) return fail(ETG_ENOTSYM, "etg_cc needs ETG_SYMMETRIC");
     if (g->n == 0) return ETG_OK;
+    if (g->comm) {
+        if (g->push && alg == ALG_BFS) return fail(ETG_EINVAL, "ETG_PUSH handles serve SSSP/CC/SSWP (BFS: destination partition)");
+        if (g->comm->device >= 0) ETG_CU(cudaSetDevice(g->comm->device));
+        return g->p.u64 ? comm_run_impl<uint64_t>(g, alg, source, label, st)
+                        : comm_run_impl<uint32_t>(g, alg, source, label, st);
+    }
     return g->p.u64 ? run_impl<uint64_t>(g, alg, source, label, st)
                     : run_impl<uint32_t>(g, alg, source, label, st);
 }
@@ -701,6 +861,120 @@ etg_status replay_impl(etg_graph *g, int alg, uint32_t source, uint32_t depth, u
     return ETG_OK;
 }
 
+// Destination partition: store what changed in the owned range into every
+// peer's copy (BFS: non-zero bitmap words; SSSP/CC/SSWP: moved labels).
+etg_status publish_impl(etg_graph *g) {
+    if (g->dpeer < 2 || g->dpeer_hi <= g->dpeer_lo) return ETG_OK;
+    PeerSet ps;
+    ps.P = g->dpeer;
+    ps.rank = g->dpeer_rank;
+    const bool bfs = g->step_alg == ALG_BFS;
+    for (uint32_t k = 0; k < kMaxPeer; ++k) ps.ptr[k] = bfs ? g->dpeer_Q[k] : g->dpeer_label[k];
+    const uint32_t *Q = reinterpret_cast<const uint32_t *>(g->ws + g->L.Q);
+    const uint32_t *snap = reinterpret_cast<const uint32_t *>(g->ws + g->L.snap);
+    if (bfs)
+        publish_kernel<true><<<g->grid_init, kBlock, 0, g->stream>>>(Q, g->step_label, snap, g->dpeer_lo,
+                                                                     g->dpeer_hi, ps);
+    else
+        publish_kernel<false><<<g->grid_init, kBlock, 0, g->stream>>>(Q, g->step_label, snap, g->dpeer_lo,
+                                                                      g->dpeer_hi, ps);
+    ETG_CU(cudaGetLastError());
+    g->step_launches += 1;
+    return ETG_OK;
+}
+
+// Base of the allocation holding d_ptr (driver API, resolved at run time: the
+// library does not link libcuda), its CUDA-IPC handle and d_ptr's offset.
+etg_status ipc_handle_of(const void *d_ptr, uint8_t *out_handle, uint64_t *out_offset) {
+    typedef CUresult (*get_attr_t)(void *, CUpointer_attribute, CUdeviceptr);
+    static get_attr_t get_attr = nullptr;
+    if (!get_attr) {
+        void *h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_GLOBAL);
+        if (h) get_attr = (get_attr_t)dlsym(h, "cuPointerGetAttribute");
+        if (!get_attr) return fail(ETG_ECUDA, "cuPointerGetAttribute unavailable (no libcuda.so.1)");
+    }
+    CUdeviceptr base = 0;
+    if (get_attr(&base, CU_POINTER_ATTRIBUTE_RANGE_START_ADDR, (CUdeviceptr)d_ptr) != CUDA_SUCCESS)
+        return fail(ETG_ECUDA, "cuPointerGetAttribute(RANGE_START_ADDR) failed");
+    cudaIpcMemHandle_t hd;
+    ETG_CU(cudaIpcGetMemHandle(&hd, (void *)base));
+    memcpy(out_handle, &hd, sizeof(hd));
+    *out_offset = (uint64_t)((CUdeviceptr)d_ptr - base);
+    return ETG_OK;
+}
+
+// Collective part of etg_load_csr on a communicator: exchange owned ranges and
+// workspace handles, check that the ranges tile [0, n), map every peer's
+// workspace (CUDA IPC; peers in this process: their pointer as is) and wire
+// the exchange of the chosen partition.  Uses slot positions 10..15 and ends
+// with a barrier.
+etg_status comm_setup(etg_graph *g, uint32_t v_lo, uint32_t v_hi) {
+    const etg::Comm &c = *g->comm;
+    etg::CommSlot &me = c.sh->slot[c.rank];
+    if (c.world > 1) {
+        etg_status rc = ipc_handle_of(g->ws, me.ipc, &me.ipc_off);
+        if (rc != ETG_OK) return rc;
+    }
+    me.ws_ptr = reinterpret_cast<uint64_t>(g->ws);
+    const uint64_t mine[6] = {g->n, v_lo, v_hi, g->L.Q, g->L.Lfull, g->push ? 1u : 0u};
+    uint64_t all[etg::kCommMaxRanks][etg::kCommVals];
+    etg_status rc = comm_gather(c, 10, mine, 6, all);
+    if (rc != ETG_OK) return rc;
+    std::string err;
+    uint32_t bounds[kMaxPeer + 1] = {};
+    for (int q = 0; q < c.world && err.empty(); ++q) {
+        if (all[q][10] != g->n) err = "ranks disagree on n";
+        else if (all[q][15] != mine[5]) err = "ranks disagree on ETG_PUSH";
+        else if (all[q][11] != (q ? all[q - 1][12] : 0ull)) err = "owned ranges must tile [0, n) in rank order";
+        else if (q && (all[q][11] & 31u)) err = "inner range bounds must be multiples of 32";
+        bounds[q] = (uint32_t)all[q][11];
+    }
+    if (err.empty() && all[c.world - 1][12] != g->n) err = "owned ranges must tile [0, n) in rank order";
+    bounds[c.world] = (uint32_t)g->n;
+    uint32_t *peer_ws[kMaxPeer] = {};
+    for (int q = 0; q < c.world && err.empty(); ++q) {
+        if (q == c.rank) {
+            peer_ws[q] = reinterpret_cast<uint32_t *>(g->ws);
+            continue;
+        }
+        const etg::CommSlot &o = c.sh->slot[q];
+        if (o.pid == getpid()) {
+            peer_ws[q] = reinterpret_cast<uint32_t *>(o.ws_ptr);    // same address space
+            continue;
+        }
+        cudaIpcMemHandle_t hd;
+        memcpy(&hd, o.ipc, sizeof(hd));
+        void *base = nullptr;
+        cudaError_t e = cudaIpcOpenMemHandle(&base, hd, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) {
+            err = std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e);
+            break;
+        }
+        g->ipc_base[q] = base;
+        peer_ws[q] = reinterpret_cast<uint32_t *>(static_cast<uint8_t *>(base) + o.ipc_off);
+    }
+    ETG_BAR(c, "load");                  // slots 10..15 read by everyone; peers mapped
+    if (!err.empty()) return fail(ETG_ENCCL, err);
+    const uint32_t P = (uint32_t)c.world;
+    for (uint32_t q = 0; q < P; ++q) {
+        uint8_t *base = reinterpret_cast<uint8_t *>(peer_ws[q]);
+        g->dpeer_Q[q] = reinterpret_cast<uint32_t *>(base + all[q][13]);
+        g->dpeer_label[q] = reinterpret_cast<uint32_t *>(base + all[q][14]);
+    }
+    if (g->push) {
+        for (uint32_t k = 0; k <= kMaxPeer; ++k) g->peer_bounds[k] = k <= P ? bounds[k] : (uint32_t)g->n;
+        for (uint32_t k = 0; k < kMaxPeer; ++k) g->peer_label[k] = k < P ? g->dpeer_label[k] : nullptr;
+        g->peer_rank = (uint32_t)c.rank;
+        g->npeer = P > 1 ? P : 0;
+    } else {
+        g->dpeer_lo = v_lo;
+        g->dpeer_hi = v_hi;
+        g->dpeer_rank = (uint32_t)c.rank;
+        g->dpeer = P;
+    }
+    return ETG_OK;
+}
+
 }  // namespace
 
 // =========================================================================== //
@@ -714,9 +988,12 @@ size_t etg_workspace_bytes(uint64_t n, uint64_t m, const etg_options *opt) {
 
 etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_row_offsets,
                         const uint32_t *d_col_idx, const uint32_t *d_weights, void *d_workspace,
-                        size_t workspace_bytes, void *stream, const etg_options *opt) {
+                        size_t workspace_bytes, void *stream, const etg_options *opt, const etg_comm *comm,
+                        uint32_t v_lo, uint32_t v_hi) {
     if (!out) return fail(ETG_EINVAL, "out is NULL");
     *out = nullptr;
+    if (comm && (v_lo > v_hi || v_hi > n)) return fail(ETG_EINVAL, "owned range [v_lo, v_hi) must lie in [0, n]");
+    if (!comm && opt && (opt->flags & ETG_PUSH)) return fail(ETG_EINVAL, "ETG_PUSH needs a communicator");
     if (!d_row_offsets || (m && !d_col_idx) || !d_workspace) return fail(ETG_EINVAL, "NULL device pointer");
     const uint32_t tune = env_tune();
     const Params p = derive(opt, tune);
@@ -742,6 +1019,16 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
     g->stream = static_cast<cudaStream_t>(stream);
     g->ws = static_cast<uint8_t *>(d_workspace);
     g->L = L;
+    g->delta_auto = p.nf_delta == ETG_SSSP_DELTA_AUTO;
+    if (comm) {
+        g->comm = const_cast<etg::Comm *>(&comm->c);
+        g->push = (flags & ETG_PUSH) != 0;
+        g->v_lo = (uint32_t)v_lo;
+        g->v_hi = (uint32_t)v_hi;
+    } else {
+        g->v_lo = 0;
+        g->v_hi = (uint32_t)n;
+    }
     g->ctl = reinterpret_cast<Ctl *>(g->ws + L.ctl);
     auto bail = [&](etg_status s) {
         etg_free(g);
@@ -749,6 +1036,8 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
     };
     int dev = 0;
     cudaError_t e;
+    if (comm && comm->c.device >= 0 && (e = cudaSetDevice(comm->c.device)) != cudaSuccess)
+        return bail(fail(ETG_ECUDA, std::string("load: ") + cudaGetErrorString(e)));
     if ((e = cudaGetDevice(&dev)) != cudaSuccess ||
         (e = cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess ||
         (e = cudaMallocHost(&g->h_ctl, sizeof(Ctl))) != cudaSuccess ||
@@ -769,6 +1058,10 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
     }
     if ((e = cudaStreamSynchronize(g->stream)) != cudaSuccess)
         return bail(fail(ETG_ECUDA, std::string("load sync: ") + cudaGetErrorString(e)));
+    if (g->comm) {
+        etg_status s = comm_setup(g, (uint32_t)v_lo, (uint32_t)v_hi);
+        if (s != ETG_OK) return bail(s);
+    }
     *out = g;
     return ETG_OK;
 }
@@ -824,8 +1117,9 @@ etg_status etg_step_begin(etg_graph *g, int alg, uint32_t source, uint32_t *d_la
     if (alg != ALG_CC && source >= g->n) return fail(ETG_EINVAL, "source >= n");
     if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "graph loaded without weights");
     if (alg == ALG_CC && !(g->flags & ETG_SYMMETRIC)) return fail(ETG_ENOTSYM, "etg_cc needs ETG_SYMMETRIC");
-    if (alg == ALG_SSSP && g->p.nf_delta == ETG_SSSP_DELTA_AUTO)   // ranks hold different edges
-        return fail(ETG_EINVAL, "step-wise runs need an explicit sssp_delta (every rank the same)");
+    if (alg == ALG_SSSP && g->delta_auto)   // each rank would derive its own Delta from its own edges
+        return fail(ETG_EINVAL, "step-wise runs need an explicit sssp_delta (every rank the same); "
+                                "communicator handles resolve auto from the global sums");
     if (g->n == 0) { *n_active = 0; return ETG_OK; }
     return g->p.u64 ? step_begin_impl<uint64_t>(g, alg, source, d_label, n_active, 0)
                     : step_begin_impl<uint32_t>(g, alg, source, d_label, n_active, 0);
@@ -858,156 +1152,6 @@ etg_status etg_step_end(etg_graph *g, etg_stats *st) {
     return ETG_OK;
 }
 
-etg_status etg_push_count(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *d_bounds,
-                          unsigned long long *d_counts) {
-    if (!g || !d_bounds || !d_counts) return fail(ETG_EINVAL, "NULL argument");
-    if (g->step_alg < 0 || g->step_alg == ALG_BFS) return fail(ETG_EINVAL, "no step-wise SSSP/CC/SSWP run in progress");
-    if (P < 1 || P > kPushMaxP || rank >= P) return fail(ETG_EINVAL, "need 1 <= P <= 64 and rank < P");
-    if (g->n == 0) return ETG_OK;
-    cudaStream_t s = g->stream;
-    ETG_CU(cudaMemsetAsync(d_counts, 0, sizeof(unsigned long long) * P, s));
-    const uint32_t *label = g->step_label;
-    uint32_t *snap = reinterpret_cast<uint32_t *>(g->ws + g->L.snap);
-    push_pack_kernel<false><<<g->grid_init, kBlock, 0, s>>>(label, snap, (uint32_t)g->n, d_bounds, P, rank,
-                                                            d_counts, nullptr);
-    ETG_CU(cudaGetLastError());
-    g->step_launches += 1;
-    return ETG_OK;
-}
-
-etg_status etg_push_pack(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *d_bounds,
-                         unsigned long long *d_cursor, uint32_t *d_pairs) {
-    if (!g || !d_bounds || !d_cursor || !d_pairs) return fail(ETG_EINVAL, "NULL argument");
-    if (g->step_alg < 0 || g->step_alg == ALG_BFS) return fail(ETG_EINVAL, "no step-wise SSSP/CC/SSWP run in progress");
-    if (P < 1 || P > kPushMaxP || rank >= P) return fail(ETG_EINVAL, "need 1 <= P <= 64 and rank < P");
-    if (g->n == 0) return ETG_OK;
-    uint32_t *snap = reinterpret_cast<uint32_t *>(g->ws + g->L.snap);
-    push_pack_kernel<true><<<g->grid_init, kBlock, 0, g->stream>>>(g->step_label, snap, (uint32_t)g->n, d_bounds,
-                                                                   P, rank, d_cursor, d_pairs);
-    ETG_CU(cudaGetLastError());
-    g->step_launches += 1;
-    return ETG_OK;
-}
-
-etg_status etg_push_apply(etg_graph *g, const uint32_t *d_pairs, uint64_t count) {
-    if (!g || (!d_pairs && count)) return fail(ETG_EINVAL, "NULL argument");
-    if (g->step_alg < 0 || g->step_alg == ALG_BFS) return fail(ETG_EINVAL, "no step-wise SSSP/CC/SSWP run in progress");
-    if (!count) return ETG_OK;
-    const unsigned blocks = (unsigned)std::min<uint64_t>((count + kBlock - 1) / kBlock, (uint64_t)g->grid_init);
-    if (g->step_alg == ALG_SSWP)
-        push_apply_kernel<ALG_SSWP><<<blocks, kBlock, 0, g->stream>>>(g->step_label, d_pairs, count);
-    else
-        push_apply_kernel<ALG_SSSP><<<blocks, kBlock, 0, g->stream>>>(g->step_label, d_pairs, count);
-    ETG_CU(cudaGetLastError());
-    g->step_launches += 1;
-    return ETG_OK;
-}
-
-etg_status etg_push_peers(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *h_bounds,
-                          uint32_t *const *h_peer_labels) {
-    if (!g) return fail(ETG_EINVAL, "NULL handle");
-    if (P == 0) {
-        g->npeer = 0;
-        return ETG_OK;
-    }
-    if (!h_bounds || !h_peer_labels) return fail(ETG_EINVAL, "NULL argument");
-    if (P > kMaxPeer || rank >= P) return fail(ETG_EINVAL, "need 1 <= P <= 8 and rank < P");
-    if (!g->p.warp) return fail(ETG_EINVAL, "the fused push exchange needs the warp expand kernel");
-    if (h_bounds[0] != 0 || h_bounds[P] != g->n) return fail(ETG_EINVAL, "bounds must run from 0 to n");
-    for (uint32_t k = 0; k < P; ++k) {
-        if (h_bounds[k] > h_bounds[k + 1]) return fail(ETG_EINVAL, "bounds must be non-decreasing");
-        if (!h_peer_labels[k]) return fail(ETG_EINVAL, "NULL peer label array");
-    }
-    for (uint32_t k = 0; k <= kMaxPeer; ++k) g->peer_bounds[k] = k <= P ? h_bounds[k] : (uint32_t)g->n;
-    for (uint32_t k = 0; k < kMaxPeer; ++k) g->peer_label[k] = k < P ? h_peer_labels[k] : nullptr;
-    g->peer_rank = rank;
-    g->npeer = P;
-    return ETG_OK;
-}
-
-etg_status etg_dest_peers(etg_graph *g, uint32_t P, uint32_t rank, const uint32_t *h_bounds,
-                          uint32_t *const *h_peer_Q, uint32_t *const *h_peer_labels) {
-    if (!g) return fail(ETG_EINVAL, "NULL handle");
-    if (P == 0) {
-        g->dpeer = 0;
-        return ETG_OK;
-    }
-    if (!h_bounds || !h_peer_Q || !h_peer_labels) return fail(ETG_EINVAL, "NULL argument");
-    if (P > kMaxPeer || rank >= P) return fail(ETG_EINVAL, "need 1 <= P <= 8 and rank < P");
-    if (h_bounds[0] != 0 || h_bounds[P] != g->n) return fail(ETG_EINVAL, "bounds must run from 0 to n");
-    for (uint32_t k = 0; k < P; ++k) {
-        if (h_bounds[k] > h_bounds[k + 1]) return fail(ETG_EINVAL, "bounds must be non-decreasing");
-        if (k > 0 && (h_bounds[k] & 31u)) return fail(ETG_EINVAL, "inner bounds must be multiples of 32");
-        if (!h_peer_Q[k] || !h_peer_labels[k]) return fail(ETG_EINVAL, "NULL peer array");
-    }
-    for (uint32_t k = 0; k < kMaxPeer; ++k) {
-        g->dpeer_Q[k] = k < P ? h_peer_Q[k] : nullptr;
-        g->dpeer_label[k] = k < P ? h_peer_labels[k] : nullptr;
-    }
-    g->dpeer_lo = h_bounds[rank];
-    g->dpeer_hi = h_bounds[rank + 1];
-    g->dpeer_rank = rank;
-    g->dpeer = P;
-    return ETG_OK;
-}
-
-etg_status etg_step_publish(etg_graph *g) {
-    if (!g || g->step_alg < 0) return fail(ETG_EINVAL, "no step-wise run in progress");
-    if (!g->dpeer) return fail(ETG_EINVAL, "etg_dest_peers not set");
-    if (g->dpeer < 2 || g->dpeer_hi <= g->dpeer_lo) return ETG_OK;
-    PeerSet ps;
-    ps.P = g->dpeer;
-    ps.rank = g->dpeer_rank;
-    const bool bfs = g->step_alg == ALG_BFS;
-    for (uint32_t k = 0; k < kMaxPeer; ++k) ps.ptr[k] = bfs ? g->dpeer_Q[k] : g->dpeer_label[k];
-    const uint32_t *Q = reinterpret_cast<const uint32_t *>(g->ws + g->L.Q);
-    const uint32_t *snap = reinterpret_cast<const uint32_t *>(g->ws + g->L.snap);
-    if (bfs)
-        publish_kernel<true><<<g->grid_init, kBlock, 0, g->stream>>>(Q, g->step_label, snap, g->dpeer_lo,
-                                                                     g->dpeer_hi, ps);
-    else
-        publish_kernel<false><<<g->grid_init, kBlock, 0, g->stream>>>(Q, g->step_label, snap, g->dpeer_lo,
-                                                                      g->dpeer_hi, ps);
-    ETG_CU(cudaGetLastError());
-    g->step_launches += 1;
-    return ETG_OK;
-}
-
-etg_status etg_ipc_handle(const void *d_ptr, uint8_t *out_handle, uint64_t *out_offset) {
-    if (!d_ptr || !out_handle || !out_offset) return fail(ETG_EINVAL, "NULL argument");
-    // base of the allocation holding d_ptr (driver API, resolved at run time:
-    // the library does not link libcuda)
-    typedef CUresult (*get_attr_t)(void *, CUpointer_attribute, CUdeviceptr);
-    static get_attr_t get_attr = nullptr;
-    if (!get_attr) {
-        void *h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_GLOBAL);
-        if (h) get_attr = (get_attr_t)dlsym(h, "cuPointerGetAttribute");
-        if (!get_attr) return fail(ETG_ECUDA, "cuPointerGetAttribute unavailable (no libcuda.so.1)");
-    }
-    CUdeviceptr base = 0;
-    if (get_attr(&base, CU_POINTER_ATTRIBUTE_RANGE_START_ADDR, (CUdeviceptr)d_ptr) != CUDA_SUCCESS)
-        return fail(ETG_ECUDA, "cuPointerGetAttribute(RANGE_START_ADDR) failed");
-    cudaIpcMemHandle_t hd;
-    ETG_CU(cudaIpcGetMemHandle(&hd, (void *)base));
-    memcpy(out_handle, &hd, sizeof(hd));
-    *out_offset = (uint64_t)((CUdeviceptr)d_ptr - base);
-    return ETG_OK;
-}
-
-etg_status etg_ipc_open(const uint8_t *handle, void **out_base) {
-    if (!handle || !out_base) return fail(ETG_EINVAL, "NULL argument");
-    cudaIpcMemHandle_t hd;
-    memcpy(&hd, handle, sizeof(hd));
-    ETG_CU(cudaIpcOpenMemHandle(out_base, hd, cudaIpcMemLazyEnablePeerAccess));
-    return ETG_OK;
-}
-
-etg_status etg_ipc_close(void *base) {
-    if (!base) return fail(ETG_EINVAL, "NULL argument");
-    ETG_CU(cudaIpcCloseMemHandle(base));
-    return ETG_OK;
-}
-
 etg_status etg_bitmap_layout(etg_graph *g, size_t *offset_bytes, uint32_t *nwords) {
     if (!g || !offset_bytes || !nwords) return fail(ETG_EINVAL, "NULL argument");
     *offset_bytes = g->L.Q;
@@ -1017,6 +1161,8 @@ etg_status etg_bitmap_layout(etg_graph *g, size_t *offset_bytes, uint32_t *nword
 
 void etg_free(etg_graph *g) {
     if (!g) return;
+    for (uint32_t q = 0; q < kMaxPeer; ++q)
+        if (g->ipc_base[q]) cudaIpcCloseMemHandle(g->ipc_base[q]);
     for (int a = 0; a < 4; ++a) {
         if (g->exec[a]) cudaGraphExecDestroy(g->exec[a]);
         if (g->graph[a]) cudaGraphDestroy(g->graph[a]);
@@ -1096,8 +1242,13 @@ etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_off, cons
         ETG_CU(cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), s));
         ETG_CU(cudaMemsetAsync(g->ws + g->L.Q, 0, 4ull * g->L.nwords, s));
         ETG_CU(cudaMemsetAsync(g->ws + g->L.recE, 0, g->L.ctl - g->L.recE, s));
+        // the reused handle sees this call's CSR: validate it like a fresh load would
+        if (g->flags & ETG_VALIDATE) {
+            rc = p.u64 ? validate_impl<uint64_t>(g) : validate_impl<uint32_t>(g);
+            if (rc != ETG_OK) return rc;
+        }
     } else {
-        rc = etg_load_csr(&g, n, m, d_off, d_col, d_w, base + o, scratch_bytes - o, stream, opt);
+        rc = etg_load_csr(&g, n, m, d_off, d_col, d_w, base + o, scratch_bytes - o, stream, opt, nullptr, 0, 0);
         if (rc != ETG_OK) return rc;
         Cached &c = cache[next_slot++ % 4];
         if (c.g) etg_free(c.g);
@@ -1110,6 +1261,46 @@ etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_off, cons
         if (e != cudaSuccess) rc = fail(ETG_ECUDA, std::string("run_host D2H: ") + cudaGetErrorString(e));
     }
     return rc;
+}
+
+// ---- communicator ---------------------------------------------------------
+etg_status etg_comm_unique_id(uint8_t *id) {
+    if (!id) return fail(ETG_EINVAL, "NULL id");
+    memset(id, 0, etg::kCommIdBytes);
+    memcpy(id, &etg::kCommMagic, 8);
+    FILE *f = fopen("/dev/urandom", "rb");
+    const size_t got = f ? fread(id + 8, 1, 24, f) : 0;
+    if (f) fclose(f);
+    if (got != 24) return fail(ETG_ENCCL, "could not read /dev/urandom");
+    return ETG_OK;
+}
+
+etg_status etg_comm_init(etg_comm **out, int rank, int world, const uint8_t *id, int device) {
+    if (!out || !id) return fail(ETG_EINVAL, "NULL argument");
+    *out = nullptr;
+    etg_comm *c = new (std::nothrow) etg_comm();
+    if (!c) return fail(ETG_ENOMEM, "host allocation failed");
+    bool bad_arg = false;
+    const std::string err = etg::comm_open(c->c, id, rank, world, device, &bad_arg);
+    if (!err.empty()) {
+        etg::comm_close(c->c);
+        delete c;
+        return fail(bad_arg ? ETG_EINVAL : ETG_ENCCL, "etg_comm_init: " + err);
+    }
+    *out = c;
+    return ETG_OK;
+}
+
+etg_status etg_comm_barrier(const etg_comm *c) {
+    if (!c) return fail(ETG_EINVAL, "NULL communicator");
+    ETG_BAR(c->c, "etg_comm_barrier");
+    return ETG_OK;
+}
+
+void etg_comm_free(etg_comm *c) {
+    if (!c) return;
+    etg::comm_close(c->c);
+    delete c;
 }
 
 const char *etg_status_str(etg_status s) {
@@ -1130,6 +1321,16 @@ const char *etg_status_str(etg_status s) {
 const char *etg_last_error(void) { return g_err.c_str(); }
 
 uint64_t etg_kernel_launches(void) { return g_launches.load(); }
+
+etg_status etg_sssp_delta(etg_graph *g, uint32_t *delta) {
+    if (!g || !delta) return fail(ETG_EINVAL, "NULL argument");
+    if (g->w) {
+        etg_status rc = resolve_delta(g);
+        if (rc != ETG_OK) return rc;
+    }
+    *delta = g->p.nf_delta;
+    return ETG_OK;
+}
 
 etg_status etg_debug_counters(etg_graph *g, uint64_t *out) {
     if (!g || !out) return fail(ETG_EINVAL, "null handle or output");

@@ -836,7 +836,7 @@ __device__ __forceinline__ void commit_peer(const Dev<OffT> &d, uint32_t *label,
 // ------------------------------------------------------------------------- //
 template <class OffT, int ALG, bool UDC, bool IDX, bool SMP>
 __global__ __launch_bounds__(kBlock) void expand_kernel(Dev<OffT> d, uint32_t cap_e) {
-    extern __shared__ __align__(16) uint8_t dyn_smem[];
+    extern __shared__ __align__(128) uint8_t dyn_smem[];
     constexpr bool kW = (ALG == ALG_SSSP || ALG == ALG_SSWP);
     constexpr bool kLab = (ALG != ALG_BFS);
     __shared__ Window<OffT> win;
@@ -1566,70 +1566,6 @@ __global__ void mark_kernel(uint32_t *Q, const uint32_t *act, uint32_t n_act) {
         atomicOr(&Q[act[k] >> 5], 1u << (act[k] & 31));
 }
 
-// ------------------------------------------------------------------------- //
-// NEXT-3 push exchange (source partition: a rank holds the out-edges of its
-// owned range, relaxations land on any vertex).  A label this rank lowered
-// (raised: SSWP) on a vertex it does not own is a proposal for the owner:
-// label != snap marks it, exactly as the scan's activation test does.
-// Owner ranges are multiples of 32 (one bitmap word, one warp-word, one
-// owner), bounds[0..P] in device memory.
-// ------------------------------------------------------------------------- //
-constexpr uint32_t kPushMaxP = 64;
-
-__device__ __forceinline__ uint32_t owner_of(const uint32_t *bounds, uint32_t P, uint32_t v) {
-    uint32_t q = 0;
-    while (q + 1 < P && v >= bounds[q + 1]) ++q;
-    return q;
-}
-
-// WRITE = false: counts[q] += proposals for owner q (counts zeroed by the host).
-// WRITE = true: append (v, label[v]) at cursor[q] (advanced atomically) and
-// refresh snap[v] -- the proposal is on its way to the owner.
-template <bool WRITE>
-__global__ __launch_bounds__(kBlock) void push_pack_kernel(const uint32_t *label, uint32_t *snap, uint32_t n,
-                                                           const uint32_t *bounds, uint32_t P, uint32_t rank,
-                                                           unsigned long long *counts, uint32_t *pairs) {
-    __shared__ unsigned long long s_cnt[kPushMaxP];
-    if (!WRITE)
-        for (uint32_t q = threadIdx.x; q < P; q += blockDim.x) s_cnt[q] = 0;
-    __syncthreads();
-    const uint32_t lane = lane_id(), lt = (1u << lane) - 1u;
-    const uint32_t lo = bounds[rank], hi = bounds[rank + 1];
-    const uint32_t nwords = (n + 31) / 32;
-    const uint32_t warps = gridDim.x * (blockDim.x >> 5);
-    for (uint32_t k = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < nwords; k += warps) {
-        const uint32_t v = k * 32 + lane;
-        if (k * 32 >= lo && k * 32 < hi) continue;          // owned word (warp-uniform)
-        uint32_t lv = 0;
-        bool moved = false;
-        if (v < n) {
-            lv = __ldcg(&label[v]);
-            moved = lv != __ldcg(&snap[v]);
-        }
-        const uint32_t b = __ballot_sync(kFull, moved);
-        if (!b) continue;
-        const uint32_t q = owner_of(bounds, P, k * 32);
-        if (!WRITE) {
-            if (lane == 0) atomicAdd(&s_cnt[q], (unsigned long long)__popc(b));
-            continue;
-        }
-        unsigned long long base = 0;
-        if (lane == 0) base = atomicAdd(&counts[q], (unsigned long long)__popc(b));
-        base = __shfl_sync(kFull, base, 0);
-        if (moved) {
-            const unsigned long long at = base + __popc(b & lt);
-            pairs[2 * at] = v;
-            pairs[2 * at + 1] = lv;
-            snap[v] = lv;
-        }
-    }
-    if (!WRITE) {
-        __syncthreads();
-        for (uint32_t q = threadIdx.x; q < P; q += blockDim.x)
-            if (s_cnt[q]) atomicAdd(&counts[q], s_cnt[q]);
-    }
-}
-
 // Fused destination-partition exchange (replaces the all-gather of owned
 // slices): the owner of [lo, hi) stores what changed in its range straight
 // into every peer's copy -- BFS: the non-zero words of its bitmap Q (no other
@@ -1657,20 +1593,6 @@ __global__ __launch_bounds__(kBlock) void publish_kernel(const uint32_t *Q, cons
         }
         for (uint32_t q = 0; q < ps.P; ++q)
             if (q != ps.rank) ps.ptr[q][i] = x;
-    }
-}
-
-// Received proposals: label[id] = min(label[id], val) (SSWP: max).  The scan
-// that follows activates every owned vertex whose label moved.
-template <int ALG>
-__global__ __launch_bounds__(kBlock) void push_apply_kernel(uint32_t *label, const uint32_t *pairs,
-                                                            unsigned long long count) {
-    const uint64_t pol = policy_keep();
-    for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < count;
-         i += (unsigned long long)gridDim.x * blockDim.x) {
-        const uint32_t u = pairs[2 * i], val = pairs[2 * i + 1];
-        if (ALG == ALG_SSWP) red_max(&label[u], val, pol);
-        else red_min(&label[u], val, pol);
     }
 }
 

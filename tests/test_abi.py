@@ -59,23 +59,27 @@ def test_workspace_bytes_monotone(L):
     c = L.etg_workspace_bytes(2000, 1_000_000, ctypes.byref(etg.Options(1, 0)))
     assert 0 < a < b < c
     # C2-sized workspace stays small next to the CSR (8 n B of col/w per edge x 16):
-    # snap, F, B, D, S, Lx (6 arrays of n words) + the bitmaps Q, V + tile_first + scan descriptors
+    # snap, F, B, D, S, Lx, Lfull (7 arrays of n words) + the bitmaps Q, V + tile_first + scan descriptors
     n, m = 1 << 22, 67_000_000
     ws = L.etg_workspace_bytes(n, m, ctypes.byref(o))
-    assert 24 * n < ws < 26 * n
+    assert 28 * n < ws < 30 * n
 
 
 def test_load_rejects_bad_arguments_without_gpu(L):
     h = ctypes.c_void_p()
     o = etg.Options(32, 0)
-    rc = L.etg_load_csr(ctypes.byref(h), 10, 5, None, None, None, None, 0, None, ctypes.byref(o))
+    rc = L.etg_load_csr(ctypes.byref(h), 10, 5, None, None, None, None, 0, None, ctypes.byref(o), None, 0, 0)
     assert rc == -1  # ETG_EINVAL before touching the device
     rc = L.etg_load_csr(ctypes.byref(h), 1 << 33, 5, ctypes.c_void_p(256), ctypes.c_void_p(256),
-                        None, ctypes.c_void_p(256), 1 << 40, None, ctypes.byref(o))
+                        None, ctypes.c_void_p(256), 1 << 40, None, ctypes.byref(o), None, 0, 0)
     assert rc == -6  # ETG_ERANGE: n > 2^32 - 2
     rc = L.etg_load_csr(ctypes.byref(h), 10, 1 << 32, ctypes.c_void_p(256), ctypes.c_void_p(256),
-                        None, ctypes.c_void_p(256), 1 << 40, None, ctypes.byref(o))
+                        None, ctypes.c_void_p(256), 1 << 40, None, ctypes.byref(o), None, 0, 0)
     assert rc == -6  # m >= 2^32 needs u64 offsets
+    push = etg.Options(32, etg.PUSH)
+    rc = L.etg_load_csr(ctypes.byref(h), 10, 5, ctypes.c_void_p(256), ctypes.c_void_p(256),
+                        None, ctypes.c_void_p(256), 1 << 40, None, ctypes.byref(push), None, 0, 10)
+    assert rc == -1  # ETG_PUSH needs a communicator
 
 
 @pytest.mark.skipif(torch.cuda.is_available(), reason="checks the no-GPU behaviour")

@@ -1,13 +1,18 @@
-"""Multi-rank path: partitioning and the exchange driver, on the CPU.
+"""Multi-rank host logic on the CPU (no GPU needed).
 
 * partition properties (every edge in exactly one part, word-aligned ranges,
-  in-edge balance);
-* the driver with P in-process ranks (LoopbackGroup) and with world_size 2
-  over gloo (torch.distributed, 127.0.0.1), each rank a test-only numpy step
-  engine (tests/etg_mock_engine.py) -- labels must equal the oracle's.
-The CUDA engine through the same driver is covered by tests/test_gpu_dist.py.
+  in-/out-edge balance);
+* the library's communicator (etg_comm_*: shared-memory rendezvous and host
+  barrier, include/etg.h), which is the control plane of the partitioned loop:
+  P threads in one process, world_size 2 over gloo (torch.distributed only
+  hands rank 0's id to rank 1, 127.0.0.1), argument errors, a missing peer
+  (timeout) and a dead peer, each reported as an error instead of a hang.
+The partitioned traversal itself (C++ loop + peer-memory kernels) is covered
+on the GPU by tests/test_gpu_dist.py.
 """
 import os
+import threading
+import time
 
 import numpy as np
 import pytest
@@ -16,31 +21,15 @@ import torch.distributed as dist
 import torch.multiprocessing as mp
 
 import graphgen as gg
-import oracle
-from etg_mock_engine import MockEngine
+import paper_conf_ipps_wangzlg19_b200 as etg
+from paper_conf_ipps_wangzlg19_b200 import _build
 from paper_conf_ipps_wangzlg19_b200 import dist as edist
 
-ALGS = {"bfs": 0, "sssp": 1, "cc": 2, "sswp": 3}
 
-
-def expected(alg, g, s):
-    off, col, w = g.numpy()
-    if alg == "bfs":
-        return oracle.bfs(off, col, s)
-    if alg == "sssp":
-        return oracle.sssp(off, col, w, s)
-    if alg == "sswp":
-        return oracle.sswp(off, col, w, s)
-    return oracle.cc(off, col)
-
-
-def make_parts(g, P):
-    bounds = edist.partition_ranges(g.off, g.col, g.n, P)
-    parts = []
-    for r in range(P):
-        loff, lcol, lw = edist.partition_csr(g.off, g.col, g.w, g.n, bounds[r], bounds[r + 1])
-        parts.append(MockEngine(loff.numpy(), lcol.numpy(), None if lw is None else lw.numpy(), g.n))
-    return bounds, parts
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    _build.build()
+    etg.lib()
 
 
 @pytest.mark.parametrize("P", [1, 2, 3, 5])
@@ -61,171 +50,106 @@ def test_partition_properties(P):
     assert seen == g.m
 
 
-@pytest.mark.parametrize("gather", [False, True])
-@pytest.mark.parametrize("alg", ["bfs", "sssp", "cc", "sswp"])
-@pytest.mark.parametrize("P", [2, 3])
-def test_loopback_driver_matches_oracle(alg, P, gather):
-    """Both exchanges: full-array all-reduce, and the all-gather of owned slices."""
-    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
-    s = gg.first_source(g)
-    bounds, parts = make_parts(g, P)
-    labels, st = edist.run_partitions(parts, edist.LoopbackGroup(), ALGS[alg], s,
-                                      bounds if gather else None)
-    np.testing.assert_array_equal(labels.numpy().view(np.uint32), expected(alg, g, s))
-    if alg == "bfs":
-        assert st.edges_processed == int(np.diff(g.off.numpy())[expected(alg, g, s) != oracle.INF].sum())
-
-
-@pytest.mark.parametrize("alg", ["bfs", "sssp", "cc", "sswp"])
-@pytest.mark.parametrize("P", [2, 3])
-def test_dest_p2p_loopback_matches_oracle(alg, P):
-    """The fused destination-partition exchange's protocol: each engine
-    publishes its owned changes into the peers' copies, no collective."""
-    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
-    s = gg.first_source(g)
-    bounds, parts = make_parts(g, P)
-    for r, p in enumerate(parts):
-        p.set_dest_peers(bounds, r, [q.q for q in parts], [q.labels for q in parts])
-    labels, st = edist.run_partitions(parts, edist.LoopbackGroup(), ALGS[alg], s, bounds, "p2p")
-    for p in parts:       # every rank holds the full result, as with the all-gather
-        np.testing.assert_array_equal(p.labels.numpy().view(np.uint32), expected(alg, g, s))
-
-
-def _gloo_worker(rank, world, port, alg, out, gather=False):
-    os.environ["MASTER_ADDR"] = "127.0.0.1"
-    os.environ["MASTER_PORT"] = str(port)
-    dist.init_process_group("gloo", rank=rank, world_size=world)
-    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
-    s = gg.first_source(g)
-    bounds = edist.partition_ranges(g.off, g.col, g.n, world)
-    loff, lcol, lw = edist.partition_csr(g.off, g.col, g.w, g.n, bounds[rank], bounds[rank + 1])
-    eng = MockEngine(loff.numpy(), lcol.numpy(), None if lw is None else lw.numpy(), g.n)
-    labels, st = edist.run_partitions([eng], edist.TorchDistGroup(), ALGS[alg], s, bounds if gather else None)
-    torch.save(labels, out + f".{rank}")
-    dist.destroy_process_group()
-
-
-@pytest.mark.parametrize("gather", [False, True])
-@pytest.mark.parametrize("alg", ["bfs", "sssp", "cc"])
-def test_gloo_world2_matches_oracle(alg, gather, tmp_path):
-    port = 29500 + (os.getpid() % 1000) + ALGS[alg] + (8 if gather else 0)
-    out = str(tmp_path / "labels")
-    mp.spawn(_gloo_worker, args=(2, port, alg, out, gather), nprocs=2, join=True)
-    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
-    exp = expected(alg, g, gg.first_source(g))
-    for r in range(2):
-        got = torch.load(out + f".{r}").numpy().view(np.uint32)
-        np.testing.assert_array_equal(got, exp)
-
-
-# --------------------------------------------------------------------------- #
-# NEXT-3: source partition + push exchange (all-to-all of proposals / dense
-# reduce onto the owners)
-# --------------------------------------------------------------------------- #
-def make_src_parts(g, P):
-    bounds = edist.partition_ranges(g.off, g.col, g.n, P, by="out")
-    parts = []
-    for r in range(P):
-        loff, lcol, lw = edist.partition_csr_src(g.off, g.col, g.w, g.n, bounds[r], bounds[r + 1])
-        parts.append(MockEngine(loff.numpy(), lcol.numpy(), None if lw is None else lw.numpy(), g.n))
-    return bounds, parts
-
-
-def owned(labels_per_rank, bounds):
-    return np.concatenate([labels_per_rank[r][bounds[r]:bounds[r + 1]] for r in range(len(bounds) - 1)])
-
-
-@pytest.mark.parametrize("P", [1, 2, 3, 5])
+@pytest.mark.parametrize("P", [1, 2, 3, 4])
 def test_source_partition_properties(P):
     g = gg.make("T12")
     bounds = edist.partition_ranges(g.off, g.col, g.n, P, by="out")
     assert bounds[0] == 0 and bounds[-1] == g.n and all(b % 32 == 0 for b in bounds[:-1])
-    off = g.off.numpy().astype(np.int64)
-    seen = 0
+    deg = np.diff(g.off.numpy())
+    tot = 0
     for r in range(P):
         lo, hi = bounds[r], bounds[r + 1]
         loff, lcol, lw = edist.partition_csr_src(g.off, g.col, g.w, g.n, lo, hi)
-        loff = loff.numpy()
-        assert loff.shape[0] == g.n + 1 and loff[-1] == lcol.shape[0]
-        deg = np.diff(loff)
-        assert np.all(deg[:lo] == 0) and np.all(deg[hi:] == 0)
-        np.testing.assert_array_equal(deg[lo:hi], np.diff(off)[lo:hi])
-        np.testing.assert_array_equal(lcol.numpy(), g.col.numpy()[off[lo]:off[hi]])
-        np.testing.assert_array_equal(lw.numpy(), g.w.numpy()[off[lo]:off[hi]])
-        seen += lcol.shape[0]
-        if P > 1:
-            assert abs((off[hi] - off[lo]) / g.m - 1 / P) < 0.05
-    assert seen == g.m
+        ldeg = np.diff(loff.numpy())
+        assert np.array_equal(ldeg[lo:hi], deg[lo:hi]) and ldeg[:lo].sum() == 0 and ldeg[hi:].sum() == 0
+        a = int(g.off[lo])
+        assert torch.equal(lcol, g.col[a:a + lcol.shape[0]].to(torch.int32))
+        assert abs(deg[lo:hi].sum() / g.m - 1 / P) < 0.05
+        tot += lcol.shape[0]
+    assert tot == g.m
 
 
-@pytest.mark.parametrize("mode", ["sparse", "dense", "auto"])
-@pytest.mark.parametrize("alg", ["sssp", "cc", "sswp"])
-@pytest.mark.parametrize("P", [2, 3])
-def test_push_loopback_matches_oracle(alg, P, mode):
-    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
-    s = gg.first_source(g)
-    bounds, parts = make_src_parts(g, P)
-    _, st, used = edist.run_push(parts, edist.LoopbackGroup(), ALGS[alg], s, bounds, list(range(P)), mode)
-    got = owned([p.labels.numpy().view(np.uint32) for p in parts], bounds)
-    np.testing.assert_array_equal(got, expected(alg, g, s))
-    if mode != "auto":
-        assert used[mode] > 0 and sum(used.values()) == used[mode]
+# --------------------------------------------------------------------------- #
+# communicator
+# --------------------------------------------------------------------------- #
+def test_comm_barrier_threads():
+    """P ranks as threads: after barrier k every rank sees all P arrivals of phase k."""
+    P, rounds = 4, 200
+    uid = etg.Comm.unique_id()
+    assert len(uid) == 128 and uid != etg.Comm.unique_id()
+    arrivals = [0] * rounds
+    lock = threading.Lock()
+    bad = []
+
+    def rank(r):
+        c = etg.Comm(r, P, uid)
+        for k in range(rounds):
+            with lock:
+                arrivals[k] += 1
+            c.barrier()
+            if arrivals[k] != P:
+                bad.append((r, k, arrivals[k]))
+        c.close()
+    ts = [threading.Thread(target=rank, args=(r,)) for r in range(P)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    assert not bad and arrivals == [P] * rounds
 
 
-@pytest.mark.parametrize("alg", ["sssp", "cc", "sswp"])
-@pytest.mark.parametrize("P", [2, 3])
-def test_push_p2p_loopback_matches_oracle(alg, P):
-    """The fused exchange's driver protocol (expand writes the owners' labels,
-    sync + barrier, scan) with the numpy engine writing peers' arrays."""
-    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
-    s = gg.first_source(g)
-    bounds, parts = make_src_parts(g, P)
-    for r, p in enumerate(parts):
-        p.set_peers(bounds, r, [q.labels for q in parts])
-    _, st, used = edist.run_push(parts, edist.LoopbackGroup(), ALGS[alg], s, bounds, list(range(P)), "p2p")
-    got = owned([p.labels.numpy().view(np.uint32) for p in parts], bounds)
-    np.testing.assert_array_equal(got, expected(alg, g, s))
-    assert used.get("p2p", 0) > 0 and used["sparse"] == used["dense"] == 0
+def test_comm_argument_errors():
+    uid = etg.Comm.unique_id()
+    with pytest.raises(etg.EtgError, match="EINVAL"):
+        etg.Comm(2, 2, uid)                               # rank >= world
+    with pytest.raises(etg.EtgError, match="EINVAL"):
+        etg.Comm(0, 9, uid)                               # world > 8
+    with pytest.raises(etg.EtgError, match="EINVAL"):
+        etg.Comm(0, 1, bytes(128))                        # not a unique id
+    c = etg.Comm(0, 1, etg.Comm.unique_id())              # world 1: nothing to wait for
+    c.barrier()
+    c.close()
 
 
-def test_push_p2p_needs_peers():
-    g = gg.make("T12")
-    bounds, parts = make_src_parts(g, 2)
-    with pytest.raises(edist.EtgError):
-        edist.run_push(parts, edist.LoopbackGroup(), ALGS["sssp"], gg.first_source(g), bounds, [0, 1], "p2p")
+def test_comm_missing_peer_times_out(monkeypatch):
+    monkeypatch.setenv("ETG_COMM_TIMEOUT_S", "1")
+    t = time.time()
+    with pytest.raises(etg.EtgError, match="ENCCL"):
+        etg.Comm(0, 2, etg.Comm.unique_id())              # rank 1 never comes
+    assert time.time() - t < 30
 
 
-def test_push_rejects_bfs():
-    g = gg.make("T12")
-    bounds, parts = make_src_parts(g, 2)
-    with pytest.raises(edist.EtgError):
-        edist.run_push(parts, edist.LoopbackGroup(), ALGS["bfs"], 0, bounds, [0, 1])
-
-
-def _gloo_push_worker(rank, world, port, alg, out, mode):
+def _gloo_worker(rank, world, port, tmp, die):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
-    s = gg.first_source(g)
-    bounds = edist.partition_ranges(g.off, g.col, g.n, world, by="out")
-    loff, lcol, lw = edist.partition_csr_src(g.off, g.col, g.w, g.n, bounds[rank], bounds[rank + 1])
-    eng = MockEngine(loff.numpy(), lcol.numpy(), None if lw is None else lw.numpy(), g.n)
-    labels, st, used = edist.run_push([eng], edist.TorchDistGroup(), ALGS[alg], s, bounds, [rank], mode)
-    torch.save((labels, bounds, used), out + f".{rank}")
-    dist.destroy_process_group()
+    c = edist.comm_from_group(rank, world)
+    for k in range(50):
+        open(os.path.join(tmp, f"r{rank}.{k}"), "w").close()
+        c.barrier()
+        for q in range(world):                            # every rank's phase-k mark is there
+            assert os.path.exists(os.path.join(tmp, f"r{q}.{k}"))
+    if die and rank == 1:
+        os._exit(0)                                       # leave without the next barrier
+    if die:
+        os.environ["ETG_COMM_TIMEOUT_S"] = "120"
+        t = time.time()
+        try:
+            c.barrier()
+            raise SystemExit(3)
+        except etg.EtgError as e:
+            assert "ENCCL" in str(e) and time.time() - t < 60
+    else:
+        c.barrier()
+    c.close()
+    open(os.path.join(tmp, f"ok{rank}"), "w").close()
 
 
-@pytest.mark.parametrize("mode", ["sparse", "dense", "auto"])
-@pytest.mark.parametrize("alg", ["sssp", "cc"])
-def test_push_gloo_world2_matches_oracle(alg, mode, tmp_path):
-    port = 31500 + (os.getpid() % 1000) + 4 * ALGS[alg] + {"sparse": 0, "dense": 1, "auto": 2}[mode]
-    out = str(tmp_path / "labels")
-    mp.spawn(_gloo_push_worker, args=(2, port, alg, out, mode), nprocs=2, join=True)
-    g = gg.make("T12") if alg != "cc" else gg.make("T12", symmetric=True, weights=False)
-    exp = expected(alg, g, gg.first_source(g))
-    res = [torch.load(out + f".{r}") for r in range(2)]
-    bounds = res[0][1]
-    got = owned([res[r][0].numpy().view(np.uint32) for r in range(2)], bounds)
-    np.testing.assert_array_equal(got, exp)
-    assert res[0][2] == res[1][2]                     # both ranks took the same exchange each iteration
+@pytest.mark.parametrize("die", [False, True])
+def test_comm_gloo_world2(tmp_path, die):
+    """world_size 2 over gloo: the id travels by torch.distributed, the barrier
+    orders the ranks; a rank that dies is detected (ENCCL), not waited for."""
+    port = 29600 + os.getpid() % 200 + (7 if die else 0)
+    mp.spawn(_gloo_worker, args=(2, port, str(tmp_path), die), nprocs=2, join=True)
+    assert os.path.exists(tmp_path / "ok0")
+    assert die or os.path.exists(tmp_path / "ok1")

@@ -1,7 +1,9 @@
 """Parity at BASELINE.json's full sizes, in the launch configuration bench.py
-times (CUDA-graph loop, K = 32, default flags): C2 (the bench workload) and
-C3 (LiveJournal-shaped, UDC on and off).  The single-threaded oracle finishes
-these in seconds, so the comparison is complete (all n labels), not sampled."""
+times (CUDA-graph loop, K = 32, default flags, SSSP with sssp_delta="auto" --
+bench.py's default schedule): C2 (the bench workload) and C3
+(LiveJournal-shaped, UDC on and off).  The paper's own SSSP schedule (Delta =
+0) is checked beside it.  The single-threaded oracle finishes these in
+seconds, so the comparison is complete (all n labels), not sampled."""
 import numpy as np
 import pytest
 import torch
@@ -21,13 +23,18 @@ def c2():
 
 
 def test_c2_bfs_sssp_sswp(c2):
+    """The bench's handle (bench.py mk(): K = 32, flags 0, sssp_delta "auto")
+    and its sources (gg.sample_sources(g, 16, 4242), the first three)."""
     off, col, w = c2.to("cpu").numpy()
-    G = to_etg(c2)
-    for s in gg.sample_sources(c2, 2, 4242):
+    G = to_etg(c2, sssp_delta="auto")
+    for s in gg.sample_sources(c2, 16, 4242)[:3]:
         np.testing.assert_array_equal(U32(G.bfs(s)[0]), oracle.bfs(off, col, s))
-        np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
+        np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s), err_msg=f"auto s={s}")
     s = gg.first_source(c2)
     np.testing.assert_array_equal(U32(G.sswp(s)[0]), oracle.sswp(off, col, w, s))
+    # the paper's schedule (Proc. 1: every improved vertex active next iteration)
+    Gp = to_etg(c2, sssp_delta=0)
+    np.testing.assert_array_equal(U32(Gp.sssp(s)[0]), oracle.sssp(off, col, w, s), err_msg="paper schedule")
 
 
 def test_c2_cc():
@@ -41,55 +48,31 @@ def test_c2_cc():
 def test_c3_lj_shaped(flags):
     g = gg.make("C3", device="cuda")
     off, col, w = g.to("cpu").numpy()
-    G = to_etg(g, flags=flags)
-    s = gg.first_source(g)
-    np.testing.assert_array_equal(U32(G.bfs(s)[0]), oracle.bfs(off, col, s))
-    np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
+    G = to_etg(g, flags=flags, sssp_delta="auto")
+    for s in [gg.first_source(g)] + gg.sample_sources(g, 16, 4242)[:1]:
+        np.testing.assert_array_equal(U32(G.bfs(s)[0]), oracle.bfs(off, col, s))
+        np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s), err_msg=f"auto s={s}")
 
 
-def test_c2_push_exchange_4way(c2):
-    """NEXT-3 at the bench size: SSSP and CC on a 4-way SOURCE partition with the
-    push exchange (auto: sparse all-to-all or dense reduce per iteration), P
-    engines on one GPU (LoopbackGroup); owned slices assembled = the oracle."""
+@pytest.mark.parametrize("exchange", ["dest", "push"])
+def test_c2_partitioned_4way(c2, exchange):
+    """The partitioned path at the bench size: 4 communicator ranks (threads,
+    one GPU), SSSP in the bench's schedule (auto Delta, resolved from the
+    global sums) and CC; owned slices concatenated = the oracle, all n."""
     from paper_conf_ipps_wangzlg19_b200 import dist as edist
-    P = 4
-
-    def run(g, alg, s):
-        bounds = edist.partition_ranges(g.off, g.col, g.n, P, by="out")
-        engs = []
-        for r in range(P):
-            loff, lcol, lw = edist.partition_csr_src(g.off, g.col, g.w, g.n, bounds[r], bounds[r + 1])
-            o, c, w, fl = etg.csr_to_device(loff, lcol, lw, device="cuda")
-            engs.append(edist.CudaEngine(etg.Graph(o, c, w, n=g.n, flags=fl, symmetric=g.symmetric)))
-        _, _, used = edist.run_push(engs, edist.LoopbackGroup(), alg, s, bounds, list(range(P)))
-        return np.concatenate([U32(e.labels)[bounds[r]:bounds[r + 1]] for r, e in enumerate(engs)]), used
-
     off, col, w = c2.to("cpu").numpy()
-    s = gg.sample_sources(c2, 1, 4242)[0]
-    got, used = run(c2, etg.SSSP, s)
-    np.testing.assert_array_equal(got, oracle.sssp(off, col, w, s))
-    assert used["sparse"] > 0 and used["dense"] > 0          # both exchanges exercised at this size
+    s = gg.sample_sources(c2, 16, 4242)[0]
+    parts = edist.local_partitions(c2.off, c2.col, c2.w, c2.n, 4, exchange=exchange, sssp_delta="auto")
+    labels, st = edist.run_local(parts, etg.SSSP, s)
+    np.testing.assert_array_equal(U32(labels), oracle.sssp(off, col, w, s))
+    if exchange == "dest":
+        labels, _ = edist.run_local(parts, etg.BFS, s)
+        np.testing.assert_array_equal(U32(labels), oracle.bfs(off, col, s))
+    for p in parts:
+        p.close()
+    del parts
     gs = gg.make("C2", device="cuda", symmetric=True, weights=False)
     soff, scol, _ = gs.to("cpu").numpy()
-    got, _ = run(gs, etg.CC, 0)
-    np.testing.assert_array_equal(got, oracle.cc(soff, scol))
-
-
-def test_c2_push_p2p_4way(c2):
-    """The fused push exchange at the bench size: 4 source partitions on one GPU,
-    each expand reducing straight into the owners' label arrays."""
-    from paper_conf_ipps_wangzlg19_b200 import dist as edist
-    P = 4
-    bounds = edist.partition_ranges(c2.off, c2.col, c2.n, P, by="out")
-    engs = []
-    for r in range(P):
-        loff, lcol, lw = edist.partition_csr_src(c2.off, c2.col, c2.w, c2.n, bounds[r], bounds[r + 1])
-        o, c, w, fl = etg.csr_to_device(loff, lcol, lw, device="cuda")
-        engs.append(edist.CudaEngine(etg.Graph(o, c, w, n=c2.n, flags=fl)))
-    for r, e in enumerate(engs):
-        e.set_peers(bounds, r, [x.labels.data_ptr() for x in engs])
-    s = gg.sample_sources(c2, 1, 4242)[0]
-    edist.run_push(engs, edist.LoopbackGroup(), etg.SSSP, s, bounds, list(range(P)), "p2p")
-    off, col, w = c2.to("cpu").numpy()
-    got = np.concatenate([U32(e.labels)[bounds[r]:bounds[r + 1]] for r, e in enumerate(engs)])
-    np.testing.assert_array_equal(got, oracle.sssp(off, col, w, s))
+    parts = edist.local_partitions(gs.off, gs.col, None, gs.n, 4, exchange=exchange, symmetric=True)
+    labels, _ = edist.run_local(parts, etg.CC, 0)
+    np.testing.assert_array_equal(U32(labels), oracle.cc(soff, scol))

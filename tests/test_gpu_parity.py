@@ -266,6 +266,27 @@ def test_run_host_matches(c1):
     np.testing.assert_array_equal(out.numpy().view(np.uint32), oracle.sssp(off, col, w, s))
     etg.run_host(etg.BFS, o, c, None, s, out, scratch)
     np.testing.assert_array_equal(out.numpy().view(np.uint32), oracle.bfs(off, col, s))
+    # the cached handle is reused for a DIFFERENT graph of the same n and m:
+    # the result must follow the new CSR, and ETG_VALIDATE must check it
+    col2 = ((col.astype(np.int64) + 1) % c1.n).astype(np.uint32)
+    c2 = torch.from_numpy(col2.view(np.int32)).pin_memory()
+    for _ in range(2):
+        etg.run_host(etg.BFS, o, c2, None, s, out, scratch, flags=etg.VALIDATE)
+        np.testing.assert_array_equal(out.numpy().view(np.uint32), oracle.bfs(off, col2, s))
+    bad = c2.clone()
+    bad[7] = c1.n + 3                                     # col >= n: same sizes, malformed
+    with pytest.raises(etg.EtgError, match="EINVALID_CSR"):
+        etg.run_host(etg.BFS, o, bad, None, s, out, scratch, flags=etg.VALIDATE)
+    # CC only with an explicit symmetry assertion (no silent SYMMETRIC)
+    with pytest.raises(etg.EtgError, match="ENOTSYM"):
+        etg.run_host(etg.CC, o, c, None, 0, out, scratch)
+    gs = gg.make("C1", symmetric=True, weights=False)
+    soff, scol, _ = gs.numpy()
+    so = torch.from_numpy(soff.astype(np.int64)).to(torch.int32).pin_memory()
+    sc = torch.from_numpy(scol.view(np.int32)).pin_memory()
+    scr = torch.empty(etg.host_scratch_bytes(gs.n, gs.m, False), dtype=torch.uint8, device="cuda")
+    etg.run_host(etg.CC, so, sc, None, 0, out, scr, symmetric=True)
+    np.testing.assert_array_equal(out.numpy().view(np.uint32), oracle.cc(soff, scol))
 
 
 def test_errors():
@@ -355,11 +376,17 @@ def test_sssp_delta_auto(c1):
     G = to_etg(c1, sssp_delta="auto")
     for s in gg.sample_sources(c1, 2, 77):
         np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
-    from paper_conf_ipps_wangzlg19_b200 import dist as edist
-    e = edist.CudaEngine(to_etg(c1, sssp_delta="auto"))   # fresh handle: Delta not resolved yet
-    with pytest.raises(etg.EtgError):
-        e.begin(etg.SSSP, 0)
-    # weights all 1: Delta = max(1, 3/8) = 1, the wave then advances one hop per iteration
+    # the rule: Delta = 6 x mean weight / mean out-degree, rounded, at least 1
+    assert G.sssp_delta() == max(1, int(6.0 * float(c1.w.double().mean()) / (c1.m / c1.n) + 0.5))
+    # the step-wise API refuses a handle loaded with auto -- also after the
+    # first SSSP resolved it (sticky): separately loaded partitions would each
+    # derive their own Delta
+    import ctypes
+    lab = torch.empty(c1.n, dtype=torch.int32, device="cuda")
+    na = ctypes.c_uint32()
+    for h in (to_etg(c1, sssp_delta="auto"), G):
+        assert etg.lib().etg_step_begin(h._h, etg.SSSP, 0, ctypes.c_void_p(lab.data_ptr()), ctypes.byref(na)) == -1
+    # weights all 1: Delta = 6 x 1 / 16 -> 1 (at least 1), the wave then advances one hop per iteration
     g1 = gg.Graph("unit", c1.n, c1.off, c1.col, torch.ones_like(c1.w))
     o1, c1_, w1 = g1.numpy()
     s = gg.first_source(c1)

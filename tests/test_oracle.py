@@ -419,3 +419,41 @@ def test_udc_slices_properties(K):
     # a shadow shorter than K is always the last of its vertex (SMP classes)
     short = np.nonzero(en - st < K)[0]
     assert np.all(en[short] == off[ids[short].astype(np.int64) + 1])
+
+
+# --------------------------------------------------------------------------- #
+# the device-side SSSP certificate used at C4 size (tests/etg_testutil.py) is
+# itself pinned here, on CPU tensors: it accepts the oracle's distances and
+# rejects every plausible wrong answer (SURVEY 8(c) O-SSSP certificate)
+# --------------------------------------------------------------------------- #
+@pytest.mark.parametrize("cfg", ["C1", "LJ-small"])
+def test_sssp_certificate_gpu_pinned(cfg):
+    import torch
+    from etg_testutil import sssp_certificate_gpu
+    g = gg.make(cfg)
+    off, col, w = g.numpy()
+    for s in [gg.first_source(g)] + gg.sample_sources(g, 1, 5):
+        d = oracle.sssp(off, col, w, s)
+        ok = torch.from_numpy(d.astype(np.int64))
+        assert sssp_certificate_gpu(g, s, ok, chunk=1 << 18) is None
+        reached = np.nonzero((d != INF) & (d > 0))[0]
+        unreached = np.nonzero(d == INF)[0]
+        rng = np.random.default_rng(s)
+        bad = []
+        for v in rng.choice(reached, 3, replace=False):
+            for delta in (+1, -1):                        # off by one either way
+                x = d.astype(np.int64).copy()
+                x[v] += delta
+                bad.append(x)
+        x = d.astype(np.int64).copy()
+        x[s] = 1                                          # source not at 0
+        bad.append(x)
+        x = d.astype(np.int64).copy()
+        x[reached[0]] = INF                               # a reached vertex reported unreached
+        bad.append(x)
+        if unreached.size:
+            x = d.astype(np.int64).copy()
+            x[unreached[0]] = int(d[reached].max())       # an unreached vertex reported reached
+            bad.append(x)
+        for x in bad:
+            assert sssp_certificate_gpu(g, s, torch.from_numpy(x), chunk=1 << 18) is not None
