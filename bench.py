@@ -197,14 +197,15 @@ def measured_peak():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def ncu_traffic(config):
-    """dram bytes per expand launch from the committed ncu --set full summary, if any."""
-    path = os.path.join(ROOT, "profiles", "expand_ncu_summary.json")
+def ncu_traffic(config, algs):
+    """dram bytes per expand launch and the algorithmic bytes of the SAME launches,
+    from the committed ncu summary of this config (profiles/r02/expand_traffic_*.json,
+    tools/traffic_summary.py), if any."""
+    path = os.path.join(ROOT, "profiles", "r02", f"expand_traffic_{config}_{'+'.join(algs)}.json")
     try:
         with open(path) as f:
             d = json.load(f)
-        c = d.get(config, {})
-        return c.get("dram_bytes_per_launch"), c.get("algorithmic_bytes_of_captured_launch")
+        return d, os.path.relpath(path, ROOT)
     except (OSError, ValueError):
         return None, None
 
@@ -459,12 +460,14 @@ def run_ours(args):
                 d["edges_processed"] += st.edges_processed
         peak, peak_src = measured_peak()
         achieved = bytes_tot / (exp_ms * 1e-3) / 1e9
-        traffic, traffic_alg = ncu_traffic(args.config)
-        roof = {"bound": "hbm", "kernel": "expand_kernel", "achieved": achieved, "peak": peak,
-                "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
-                "traffic_note": ("dram read+write bytes of one ncu --set full capture of the largest BFS "
-                                 "expand launch (profiles/expand_ncu_summary.json); algorithmic bytes of "
-                                 f"that launch: {traffic_alg}") if traffic else None,
+        tr, tr_path = ncu_traffic(args.config, algs)
+        roof = {"bound": "hbm", "kernel": "expand_warp_kernel", "achieved": achieved, "peak": peak,
+                "unit": "GB/s", "frac": achieved / peak,
+                "traffic": tr["dram_bytes_per_launch"] if tr else None,
+                "traffic_note": (f"ncu dram read+write bytes per expand launch, mean over all {tr['launches']} "
+                                 f"expand launches of one call per algorithm ({tr_path}); algorithmic bytes per "
+                                 f"launch of those same launches: {tr['alg_bytes_per_launch']:.0f} "
+                                 f"(dram/algorithmic = {tr['dram_over_alg']:.2f})") if tr else None,
                 "peak_source": peak_src,
                 "algorithmic_bytes_per_launch": bytes_tot / max(1, launches_p),
                 "avg_launch_ms": exp_ms / max(1, launches_p),

@@ -36,6 +36,8 @@ def stale() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    if os.environ.get("ETG_LIB_PATH") and not force:
+        return LIB                      # a prebuilt library (A/B experiments): never rebuilt
     if not force and not stale():
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"

@@ -16,13 +16,17 @@ ap.add_argument("--algs", default="bfs")
 ap.add_argument("--K", type=int, default=32)
 ap.add_argument("--flags", type=int, default=etg.HOST_LOOP)
 ap.add_argument("--repeat", type=int, default=1)
+ap.add_argument("--sssp-delta", default="auto")
+ap.add_argument("--json", default=None, help="write per-call statistics (for the algorithmic bytes)")
 a = ap.parse_args()
 dev = torch.device("cuda:0")
 algs = a.algs.split(",")
 g = gg.make(a.config, device=dev, weights="sssp" in algs)
 src = gg.sample_sources(g, 1, 4242)[0]
 o, c, w, fl = etg.csr_to_device(g.off, g.col, g.w, device=dev)
-G = etg.Graph(o, c, w, n=g.n, K=a.K, flags=a.flags | fl)
+G = etg.Graph(o, c, w, n=g.n, K=a.K, flags=a.flags | fl, sssp_delta=a.sssp_delta)
+import json  # noqa: E402
+calls = []
 for _ in range(a.repeat):
     for alg in algs:
         if alg == "cc":
@@ -33,3 +37,8 @@ for _ in range(a.repeat):
         else:
             _, st = G.run({"bfs": etg.BFS, "sssp": etg.SSSP, "sswp": etg.SSWP}[alg], src)
         print(alg, st.asdict())
+        calls.append({"alg": alg, **st.asdict()})
+if a.json:
+    with open(a.json, "w") as f:
+        json.dump({"config": a.config, "K": a.K, "flags": a.flags, "sssp_delta": a.sssp_delta, "source": src,
+                   "calls": calls}, f)
