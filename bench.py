@@ -220,6 +220,30 @@ def build_workload(cfg, device, algs):
     return g, gs
 
 
+class pinned_core:
+    """Run the oracle pinned to one host core (single-threaded,
+    one core), restoring the previous affinity afterwards."""
+
+    def __enter__(self):
+        self.old = os.sched_getaffinity(0)
+        self.core = max(self.old)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.old)
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown CPU"
+
+
 def oracle_leg(cfg, algs, nsrc, seed, budget_s=25.0, g=None, gs=None):
     """Time the CPU oracle on a bounded sample: the algorithms of one step, from
     as many sources as fit in ``budget_s`` (at least one).  Returns (edges, seconds, sample)."""
@@ -240,14 +264,15 @@ def oracle_leg(cfg, algs, nsrc, seed, budget_s=25.0, g=None, gs=None):
     while True:
         s = srcs[k % len(srcs)]
         for a in algs:
-            t = time.perf_counter()
-            if a == "bfs":
-                lab = oracle.bfs(off, col, s)
-            elif a == "sssp":
-                lab = oracle.sssp(off, col, w, s)
-            else:
-                lab = oracle.cc(soff, scol)
-            secs += time.perf_counter() - t
+            with pinned_core():
+                t = time.perf_counter()
+                if a == "bfs":
+                    lab = oracle.bfs(off, col, s)
+                elif a == "sssp":
+                    lab = oracle.sssp(off, col, w, s)
+                else:
+                    lab = oracle.cc(soff, scol)
+                secs += time.perf_counter() - t
             if a == "cc":
                 edges += int(scol.shape[0])
             else:
@@ -301,14 +326,15 @@ def run_reference(args):
         s = srcs[(i // len(algs)) % len(srcs)]
         if i < args.warmup and i > 0:
             continue                       # nothing to warm on the CPU beyond one call
-        t = time.perf_counter()
-        if a == "bfs":
-            lab = oracle.bfs(off, col, s)
-        elif a == "sssp":
-            lab = oracle.sssp(off, col, w, s)
-        else:
-            lab = oracle.cc(soff, scol)
-        dt = time.perf_counter() - t
+        with pinned_core():
+            t = time.perf_counter()
+            if a == "bfs":
+                lab = oracle.bfs(off, col, s)
+            elif a == "sssp":
+                lab = oracle.sssp(off, col, w, s)
+            else:
+                lab = oracle.cc(soff, scol)
+            dt = time.perf_counter() - t
         if i < args.warmup:
             continue
         secs += dt
@@ -325,7 +351,8 @@ def run_reference(args):
                    "n": g.n, "m": g.m},
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
                          "sample": f"one oracle call per step, rotating {'/'.join(algs)} and sources: "
-                                   f"{counts} calls on {args.config}"},
+                                   f"{counts} calls on {args.config}; single-threaded C oracle (gcc -O3) pinned "
+                                   f"to 1 of {os.cpu_count()} host cores ({cpu_model()})"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -525,7 +552,8 @@ def run_ours(args):
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         e, secs, sample = oracle_leg(args.config, algs, args.sources, 4242, budget_s=12.0, g=g, gs=gs)
         cpu = {"value": e / secs / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"{sample} on {args.config} (single-threaded C oracle, {os.cpu_count()} host cores present)"}
+               "sample": f"{sample} on {args.config} (single-threaded C oracle, gcc -O3, pinned to 1 of "
+                         f"{os.cpu_count()} host cores, {cpu_model()})"}
 
     if rank == 0:
         line = {
@@ -538,7 +566,9 @@ def run_ours(args):
                                          else "paper (Proc. 1)"),
                        "sources": len(sources),
                        "l2": "flushed (256 MiB write) before every traversal call; col/w 4 B x m each > 126 MB L2",
-                       "parallelism": f"{world} independent replica(s), own sources per rank"},
+                       "parallelism": f"{world} independent replica(s), own sources per rank",
+                       "sha256": {g.name + "+w" if g.w is not None else g.name: g.sha256(),
+                                  **({gs.name: gs.sha256()} if gs is not None else {})}},
             "per_alg": per_alg,
             "roofline": roof,
             "cpu_baseline": cpu,

@@ -31,10 +31,11 @@ _lib = None
 
 
 def build(force: bool = False) -> str:
-    """Compile oracle.c into _oracle.so with gcc (-O2, single-threaded)."""
+    """Compile oracle.c into _oracle.so with gcc (-O3, single-threaded; no
+    -march=native: the library built here also runs on the GPU box's host CPU)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O2", "-std=c99", "-shared", "-fPIC", _SRC, "-o", tmp])
+        subprocess.check_call(["gcc", "-O3", "-std=c99", "-shared", "-fPIC", _SRC, "-o", tmp])
         os.replace(tmp, _LIB)
     return _LIB
 

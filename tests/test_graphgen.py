@@ -115,3 +115,34 @@ def test_galois_gr_roundtrip(tmp_path):
         f.truncate(40)
     with pytest.raises(ValueError):
         gr.read_gr(p)
+
+
+def _golden_sha():
+    import json
+    import os
+    return json.load(open(os.path.join(os.path.dirname(__file__), "golden", "config_sha256.json")))
+
+
+@pytest.mark.parametrize("cfg", ["T12", "C1", "LJ-small"])
+def test_config_sha256_pinned(cfg):
+    """Input provenance: the CSR of each small config is pinned by
+    its SHA-256 (tests/golden/config_sha256.json, written by tools/config_sha.py)."""
+    gold = _golden_sha()
+    g = gg.make(cfg)
+    assert gold[cfg + "+w"] == {"n": g.n, "m": g.m, "sha256": g.sha256()}
+    s = gg.make(cfg, symmetric=True, weights=False)
+    assert gold[cfg + "-sym"] == {"n": s.n, "m": s.m, "sha256": s.sha256()}
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("cfg", ["T14", "C1", "LJ-small"])
+def test_generator_cpu_equals_cuda(cfg):
+    """The same integer arithmetic on the GPU gives the same graphs, bit for bit
+    (graphgen module doc): CUDA-built CSR = the CPU-built one = the pinned hash."""
+    gold = _golden_sha()
+    for sym in (False, True):
+        gc = gg.make(cfg, device="cpu", symmetric=sym, weights=not sym)
+        gd = gg.make(cfg, device="cuda", symmetric=sym, weights=not sym)
+        assert torch.equal(gc.off, gd.off.cpu()) and torch.equal(gc.col, gd.col.cpu())
+        assert (gc.w is None) == (gd.w is None) and (gc.w is None or torch.equal(gc.w, gd.w.cpu()))
+        assert gd.sha256() == gold[cfg + ("-sym" if sym else "+w")]["sha256"]
