@@ -11,6 +11,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <dlfcn.h>
+#include <nvtx3/nvToolsExt.h>   // header-only: ranges cost nothing unless a tool is attached
 
 #include <algorithm>
 #include <atomic>
@@ -598,7 +599,7 @@ etg_status resolve_delta(etg_graph *g) {
     unsigned long long wsum = 0;
     if (g->m && g->w) {
         ETG_CU(cudaMemsetAsync(&g->ctl->reached_e, 0, sizeof(unsigned long long), g->stream));
-        weight_sum_kernel<<<g->grid_init, kBlock, 0, g->stream>>>(g->w, g->m, g->ctl);
+        weight_sum_kernel<<<g->num_sms * 8, kBlock, 0, g->stream>>>(g->w, g->m, g->ctl);
         ETG_CU(cudaGetLastError());
         ETG_CU(cudaMemcpyAsync(&g->h_ctl->reached_e, &g->ctl->reached_e, sizeof(unsigned long long),
                                cudaMemcpyDeviceToHost, g->stream));
@@ -731,7 +732,20 @@ etg_status comm_run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *out, 
     return ETG_OK;
 }
 
+etg_status run_checked(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stats *st);
+
+// One traversal call, bracketed by an NVTX range named after the algorithm
+// (and "/comm" for a communicator handle) for timeline tools.
 etg_status run(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stats *st) {
+    static const char *names[2][4] = {{"etg_bfs", "etg_sssp", "etg_cc", "etg_sswp"},
+                                      {"etg_bfs/comm", "etg_sssp/comm", "etg_cc/comm", "etg_sswp/comm"}};
+    nvtxRangePushA(names[g && g->comm ? 1 : 0][alg & 3]);
+    const etg_status rc = run_checked(g, alg, source, label, st);
+    nvtxRangePop();
+    return rc;
+}
+
+etg_status run_checked(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stats *st) {
     if (!g || !label) return fail(ETG_EINVAL, "null handle or label pointer");
     if (alg != ALG_CC && source >= g->n) return fail(ETG_EINVAL, "source >= n");
     if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "graph loaded without weights");
@@ -1050,8 +1064,11 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
         return bail(fail(ETG_ECUDA, std::string("load: ") + cudaGetErrorString(e)));
     }
     g->tune = tune;
-    g->grid_scan = g->num_sms * 4;
-    g->grid_init = g->num_sms * 8;
+    // no more scan CTAs than scan tiles, no more init CTAs than 256-vertex
+    // blocks: a small graph does not launch hundreds of CTAs that exit at once
+    const uint64_t nscan = (n + kScanV - 1) / kScanV, ninit = (std::max<uint64_t>(n, L.nwords) + kBlock - 1) / kBlock;
+    g->grid_scan = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)g->num_sms * 4, nscan));
+    g->grid_init = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)g->num_sms * 8, ninit));
     if (flags & ETG_VALIDATE) {
         etg_status s = p.u64 ? validate_impl<uint64_t>(g) : validate_impl<uint32_t>(g);
         if (s != ETG_OK) return bail(s);
