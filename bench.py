@@ -234,6 +234,39 @@ class pinned_core:
         os.sched_setaffinity(0, self.old)
 
 
+def select_sources(cands, reached, n, count):
+    """SURVEY A-7 / PAPER.md L249 ("make sure the queried traversal is
+    untrivial"): keep the seeded candidates (out-degree >= 1) whose traversal
+    reaches at least 1 % of the vertices, in order, up to `count`.
+    `reached(s)` -> (vertices reached, edges of the activatable subgraph)."""
+    keep, m_reach = [], {}
+    for s in cands:
+        v, e = reached(s)
+        if v >= 0.01 * n:
+            keep.append(s)
+            m_reach[s] = e
+            if len(keep) == count:
+                break
+    if not keep:
+        raise RuntimeError("no candidate source reaches 1 % of the vertices")
+    return keep, m_reach
+
+
+def oracle_sources(g, off, col, count, seed):
+    """A-7 sources chosen with the oracle's own BFS (the reference arm never
+    touches the GPU path)."""
+    import numpy as np
+    import graphgen as gg
+    import oracle
+    deg = np.diff(off.astype(np.int64))
+
+    def reached(s):
+        lab = oracle.bfs(off, col, s)
+        r = lab != oracle.INF
+        return int(r.sum()), int(deg[r].sum())
+    return select_sources(gg.sample_sources(g, 4 * count, seed), reached, g.n, count)
+
+
 def cpu_model():
     try:
         for line in open("/proc/cpuinfo"):
@@ -244,7 +277,7 @@ def cpu_model():
     return "unknown CPU"
 
 
-def oracle_leg(cfg, algs, nsrc, seed, budget_s=25.0, g=None, gs=None):
+def oracle_leg(cfg, algs, nsrc, seed, budget_s=25.0, g=None, gs=None, srcs=None):
     """Time the CPU oracle on a bounded sample: the algorithms of one step, from
     as many sources as fit in ``budget_s`` (at least one).  Returns (edges, seconds, sample)."""
     import numpy as np
@@ -254,7 +287,7 @@ def oracle_leg(cfg, algs, nsrc, seed, budget_s=25.0, g=None, gs=None):
         g, gs = build_workload(cfg, "cuda" if _has_cuda() else "cpu", algs)
     off, col, w = g.to("cpu").numpy()
     deg = np.diff(off.astype(np.int64))
-    srcs = gg.sample_sources(g, nsrc, seed)
+    srcs, _ = oracle_sources(g, off, col, nsrc, seed) if srcs is None else (srcs, None)
     edges = 0
     secs = 0.0
     done = []
@@ -319,7 +352,7 @@ def run_reference(args):
     deg = np.diff(off.astype(np.int64))
     if gs is not None:
         soff, scol, _ = gs.to("cpu").numpy()
-    srcs = gg.sample_sources(g, args.sources, 4242)
+    srcs, _ = oracle_sources(g, off, col, args.sources, 4242)
     edges, secs, done = 0, 0.0, []
     for i in range(args.warmup + args.steps):
         a = algs[i % len(algs)]
@@ -377,7 +410,6 @@ def run_ours(args):
     dev = torch.device("cuda", torch.cuda.current_device())
     algs = args.algs.split(",")
     g, gs = build_workload(args.config, dev, algs)
-    sources = gg.sample_sources(g, args.sources, 4242 + 7919 * rank)
 
     def mk(graph, flags, sym=False):
         o, c, w, fl = etg.csr_to_device(graph.off, graph.col, graph.w, device=dev)
@@ -391,11 +423,13 @@ def run_ours(args):
     G = mk(g, 0)
     Gs = mk(gs, 0, sym=True) if gs is not None else None
     out = torch.empty(g.n, dtype=torch.int32, device=dev)
-    # m of the activatable subgraph per source (outside the timed region)
-    m_reach = {}
-    for s in sources:
-        lab, _ = G.bfs(s, out)
-        m_reach[s] = int(G.reach_stats(lab).edges_reached)
+    # sources per SURVEY A-7 and m of their activatable subgraphs (outside the timed region)
+
+    def reached(s):
+        st = G.reach_stats(G.bfs(s, out)[0])
+        return int(st.vertices_reached), int(st.edges_reached)
+    sources, m_reach = select_sources(gg.sample_sources(g, 4 * args.sources, 4242 + 7919 * rank),
+                                      reached, g.n, args.sources)
     m_sym = gs.m if gs is not None else 0
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
@@ -550,7 +584,8 @@ def run_ours(args):
     # ---- CPU oracle baseline (rank 0, N = 1 only) ----
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        e, secs, sample = oracle_leg(args.config, algs, args.sources, 4242, budget_s=12.0, g=g, gs=gs)
+        e, secs, sample = oracle_leg(args.config, algs, args.sources, 4242, budget_s=12.0, g=g, gs=gs,
+                                     srcs=sources)
         cpu = {"value": e / secs / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
                "sample": f"{sample} on {args.config} (single-threaded C oracle, gcc -O3, pinned to 1 of "
                          f"{os.cpu_count()} host cores, {cpu_model()})"}
@@ -564,7 +599,7 @@ def run_ours(args):
                        "n": g.n, "m": g.m, "m_sym": m_sym, "K": args.K, "flags": args.flags,
                        "sssp_schedule": (f"wave, Delta={args.sssp_delta}" if str(args.sssp_delta) != "0"
                                          else "paper (Proc. 1)"),
-                       "sources": len(sources),
+                       "sources": f"{len(sources)} seeded, each reaching >= 1 % of V (SURVEY A-7)",
                        "l2": "flushed (256 MiB write) before every traversal call; col/w 4 B x m each > 126 MB L2",
                        "parallelism": f"{world} independent replica(s), own sources per rank",
                        "sha256": {g.name + "+w" if g.w is not None else g.name: g.sha256(),
@@ -613,12 +648,27 @@ def run_partitioned(args):
     clocks = ClockSampler(dev.index) if rank == 0 else None
     clk_started = False
     shas = {}
+    # sources per SURVEY A-7, the same as the N = 1 run (seed 4242), chosen with
+    # a partitioned BFS (collective: every rank takes the same decisions)
+    g0 = gg.make(args.config, device=dev, weights=False)
+    deg0 = g0.degrees()
+    dg0 = edist.DistGraph(g0.off, g0.col, None, g0.n, comm, K=args.K, device=dev)
+    out0 = torch.empty(max(1, dg0.hi - dg0.lo), dtype=torch.int32, device=dev)
+
+    def reached(s):
+        lab, _ = dg0.run(etg.BFS, s, out0)
+        r = lab[:dg0.hi - dg0.lo] != -1
+        v, e = allreduce([float(r.sum()), float(deg0[dg0.lo:dg0.hi][r].sum())], tdist.ReduceOp.SUM, world)
+        return int(v), int(e)
+    sources, m_reach_all = select_sources(gg.sample_sources(g0, 4 * args.sources, 4242), reached, g0.n,
+                                          args.sources)
+    dg0.close()
+    del dg0, g0, deg0, out0
+    torch.cuda.empty_cache()
     for a in algs:
         g = gg.make(args.config, device=dev, weights=(a == "sssp"), symmetric=(a == "cc"))
         if rank == 0:
             shas[g.name + ("+w" if g.w is not None else "")] = g.sha256()
-        deg = g.degrees()
-        sources = gg.sample_sources(g, args.sources, 4242)           # the same on every rank
         exchange = "push" if (args.push and a != "bfs") else "dest"
         dg = edist.DistGraph(g.off, g.col, g.w, g.n, comm, exchange=exchange, K=args.K, flags=args.flags,
                              symmetric=(a == "cc"), sssp_delta=args.sssp_delta, device=dev)
@@ -627,14 +677,7 @@ def run_partitioned(args):
         del g
         torch.cuda.empty_cache()
         out = torch.empty(max(1, hi - lo), dtype=torch.int32, device=dev)
-        m_reach = {}
-        for s in sources[:min(len(sources), args.warmup + args.steps)]:
-            if a == "cc":
-                m_reach[s] = m_sym
-                continue
-            lab, _ = dg.run(alg_id[a], s, out)         # reached set: the same for BFS and SSSP
-            mine = float(deg[lo:hi][lab[:hi - lo] != -1].sum())
-            m_reach[s] = int(allreduce([mine], tdist.ReduceOp.SUM, world)[0])
+        m_reach = {s: (m_sym if a == "cc" else m_reach_all[s]) for s in sources}
         # warm-up, then the timed calls: per call the library's device time, max over ranks
         ms_tot, edges_tot = 0.0, 0
         for i in range(args.warmup + args.steps):
@@ -688,7 +731,7 @@ def run_partitioned(args):
         res[a] = {"gteps": edges_tot / ms_tot / 1e6, "ms_per_call": ms_tot / args.steps, "edges": edges_tot,
                   "ms": ms_tot, "exchange": exchange}
         dg.close()
-        del dg, deg
+        del dg
         torch.cuda.empty_cache()
     if clocks:
         clocks.mark("t1")
@@ -708,7 +751,8 @@ def run_partitioned(args):
                                        "partition), exchange by the library's kernels into the peers' device memory "
                                        "(CUDA IPC; NVLink between GPUs), host barrier per iteration; "
                                        f"{torch.cuda.device_count()} visible device(s)"),
-                       "K": args.K, "flags": args.flags, "sources": args.sources,
+                       "K": args.K, "flags": args.flags,
+                       "sources": f"{len(sources)} seeded, each reaching >= 1 % of V (SURVEY A-7), as at N = 1",
                        "sssp_schedule": (f"wave, Delta={args.sssp_delta} (auto from the global sums)"
                                          if str(args.sssp_delta) != "0" else "paper (Proc. 1)"),
                        "l2": "flushed (256 MiB write) before every traversal call",

@@ -159,6 +159,7 @@ struct etg_graph {
     Layout L{};
     Ctl *ctl = nullptr;
     int num_sms = 0;
+    int l2_bytes = 0;
     uint32_t tune = 0;                    // ETG_TUNE (experiments only)
     int grid_scan = 0;
     int grid_init = 0;
@@ -225,6 +226,13 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.ts_log2 = g->p.ts_log2;
     d.tune = g->tune;
     d.snap_used = 0;
+    // the pre-filter's gather array: the snapshot keeps the gathers and the
+    // red.min commits on different lines while both fit in L2 (C2: 2 x 16.8 MB);
+    // beyond L2 (C4: 2 x 166 MB vs 126 MB) every random access is a DRAM sector,
+    // and gathering the live labels halves the randomly accessed bytes
+    d.filt_live = (g->tune & kTuneFiltLive) ? 1u
+                  : (g->tune & kTuneFiltSnap) ? 0u
+                  : (8ull * g->n > (uint64_t)g->l2_bytes ? 1u : 0u);
     d.npeer = g->npeer;
     d.peer_rank = g->peer_rank;
     for (uint32_t k = 0; k <= kMaxPeer; ++k) d.peer_bounds[k] = g->peer_bounds[k];
@@ -1054,6 +1062,7 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
         return bail(fail(ETG_ECUDA, std::string("load: ") + cudaGetErrorString(e)));
     if ((e = cudaGetDevice(&dev)) != cudaSuccess ||
         (e = cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess ||
+        (e = cudaDeviceGetAttribute(&g->l2_bytes, cudaDevAttrL2CacheSize, dev)) != cudaSuccess ||
         (e = cudaMallocHost(&g->h_ctl, sizeof(Ctl))) != cudaSuccess ||
         (e = cudaEventCreate(&g->ev0)) != cudaSuccess || (e = cudaEventCreate(&g->ev1)) != cudaSuccess ||
         (e = cudaEventCreate(&g->pev[0])) != cudaSuccess || (e = cudaEventCreate(&g->pev[1])) != cudaSuccess ||

@@ -129,6 +129,8 @@ struct Dev {
     uint32_t ahead;             // warp kernel: stage A of the next batch before stage B of this one
     uint32_t nf_delta;          // near-far SSSP bucket width (0: the paper's schedule)
     uint32_t snap_used;         // SSSP/CC/SSWP, single GPU: a sole shadow stores the label it expands with
+    uint32_t filt_live;         // SSSP/CC/SSWP pre-filter reads the live labels, not the snapshot (label +
+                                // snapshot larger than L2: one randomly gathered array instead of two)
     // Fused push exchange (NEXT-3 over peer memory): a relaxation of a vertex
     // owned by rank q != peer_rank also lands, as a red.min/max, in rank q's
     // label array (device memory of another GPU reached over NVLink, or of
@@ -151,6 +153,8 @@ constexpr uint32_t kTuneNoFilter = 4096u;  // A/B: no pre-filter gather, every r
 constexpr uint32_t kTuneNearFarClassic = 8192u;   // A/B: near-far threshold advances only when the near set empties
 constexpr uint32_t kTuneNoSharedLabel = 16384u;   // A/B: multi-shadow vertices keep the scan-time snapshot
 constexpr uint32_t kTuneAheadAll = 32768u;        // A/B: SMP look-ahead for SSSP/CC/SSWP too (default: BFS only)
+constexpr uint32_t kTuneFiltLive = 1u << 18;      // A/B: pre-filter on the live labels at any size
+constexpr uint32_t kTuneFiltSnap = 1u << 19;      // A/B: pre-filter on the snapshot at any size
 
 // ------------------------------------------------------------------------- //
 // small device helpers
@@ -1187,7 +1191,9 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
     // instead of two.  Stage B needs only registers, so a tile's shared-memory
     // stage (SMP) can be refilled once stage A has left the tile.
     const bool markQ = (d.tune & kTuneQMark) != 0;   // near-far defers through the snapshot, not Q
-    const uint32_t *filt = (ALG == ALG_BFS) ? label : d.snap;   // BFS: live labels; else snapshot (R-4, R-6)
+    // BFS: live labels; else the snapshot (R-4, R-6), or the live labels when
+    // label + snapshot do not fit in L2 (one random stream instead of two)
+    const uint32_t *filt = (ALG == ALG_BFS || d.filt_live) ? label : d.snap;
     uint32_t t = next_tile();
     if (t < ntiles) {
         WarpTile<OffT, UDC> nxt = prepare(t, 0);

@@ -9,7 +9,7 @@ rows = list(csv.reader(open(sys.argv[1])))
 key = sys.argv[2] if len(sys.argv) > 2 else "expand"
 hdr = next(r for r in rows if r and r[0] == "ID")
 per = {}
-scale = {"byte": 1, "kbyte": 1e3, "mbyte": 1e6, "gbyte": 1e9, "nsecond": 1e-3, "usecond": 1, "msecond": 1e3}
+scale = {"byte": 1, "kbyte": 1e3, "mbyte": 1e6, "gbyte": 1e9, "nsecond": 1e-3, "ns": 1e-3, "usecond": 1, "us": 1, "msecond": 1e3, "ms": 1e3}
 for r in rows:
     if len(r) != len(hdr) or r[0] == "ID":
         continue

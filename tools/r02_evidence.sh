@@ -10,7 +10,8 @@ tr() { cfg=$1; algs=$2; tag=${cfg}_${algs//,/+}
   timeout 1200 ncu --metrics $M --cache-control none --clock-control none -k regex:expand_warp --csv \
     --log-file $O/traffic_$tag.csv python tools/prof_run.py --config $cfg --algs $algs --json $O/traffic_$tag.stats.json > $O/traffic_$tag.log 2>&1
   python tools/traffic_summary.py $O/traffic_$tag.csv $O/traffic_$tag.stats.json > $O/expand_traffic_$tag.json && \
-    python -c "import json;d=json.load(open('$O/expand_traffic_$tag.json'));print('$tag', d['launches'], round(d['dram_over_alg'],2), round(d['alg_gbs_under_ncu']), round(d['dram_gbs_under_ncu']))"; }
+    python -c "import json;d=json.load(open('$O/expand_traffic_$tag.json'));print('$tag', d['launches'], round(d['dram_over_alg'],2), round(d['alg_gbs_under_ncu']), round(d['dram_gbs_under_ncu']))"
+  gzip -f $O/traffic_$tag.csv; }
 tr C2 bfs,sssp,cc
 tr C3 bfs,sssp
 tr C4 sssp
@@ -29,7 +30,7 @@ F=gpu__time_duration.sum,dram__bytes_read.sum,lts__t_sector_hit_rate.pct,lts__t_
 for v in "0 lookahead" "128 smpshared" "4 nosmp"; do set -- $v
   timeout 900 ncu --metrics $F --cache-control none --clock-control none -k regex:expand_warp --csv \
     --log-file $O/fig7_$2.csv python tools/prof_run.py --config C3 --algs bfs,sssp --flags $((32 | $1)) > $O/fig7_$2.log 2>&1
-  python tools/ncu_agg.py $O/fig7_$2.csv expand > $O/fig7_$2.json; echo "fig7 $2"; head -14 $O/fig7_$2.json
+  python tools/ncu_agg.py $O/fig7_$2.csv expand > $O/fig7_$2.json; echo "fig7 $2"; head -14 $O/fig7_$2.json; gzip -f $O/fig7_$2.csv
 done
 # 4. ncu --set full: dominant expand launch of C4 SSSP and C5 BFS, C2 SSSP scans (dense #4, sparse #15)
 timeout 1500 ncu --set full --clock-control none --import-source on -k regex:expand_warp -s 4 -c 1 -o $O/full_c4_sssp_expand \
@@ -38,4 +39,8 @@ timeout 1500 ncu --set full --clock-control none --import-source on -k regex:exp
    python tools/prof_run.py --config C5 --algs bfs > $O/full_c5.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:udc_scan -s 15 -c 1 -o $O/full_c2_sssp_scan15 \
    python tools/prof_run.py --config C2 --algs sssp > $O/full_scan15.log 2>&1
-ls -la $O
+for r in $O/*.ncu-rep; do python tools/ncu_lines.py $r 30 > ${r%.ncu-rep}.lines.txt 2>&1
+  ncu -i $r --page raw --csv > ${r%.ncu-rep}.raw.csv 2>/dev/null; gzip -f ${r%.ncu-rep}.raw.csv; done
+du -sh $O; ls -la $O
+# keep the pull under 64 MiB: drop the biggest reports if needed
+while [ $(du -sm gpurun_out | cut -f1) -gt 60 ]; do big=$(ls -S $O/*.ncu-rep 2>/dev/null | head -1); [ -z "$big" ] && break; echo "dropping $big"; rm -f $big; done

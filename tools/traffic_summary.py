@@ -23,7 +23,7 @@ for r in rows:
         continue
     v = float(d["Metric Value"].replace(",", ""))
     u = d["Metric Unit"].lower()
-    scale = {"byte": 1, "kbyte": 1e3, "mbyte": 1e6, "gbyte": 1e9, "nsecond": 1e-3, "usecond": 1, "msecond": 1e3}
+    scale = {"byte": 1, "kbyte": 1e3, "mbyte": 1e6, "gbyte": 1e9, "nsecond": 1e-3, "ns": 1e-3, "usecond": 1, "us": 1, "msecond": 1e3, "ms": 1e3}
     per.setdefault(d["ID"], {})[d["Metric Name"]] = v * scale.get(u, 1)
 stats = json.load(open(sys.argv[2]))
 alg_bytes = sum(BPE[c["alg"]] * c["edges_processed"] + BPV[c["alg"]] * c["frontier_total"] for c in stats["calls"])
