@@ -1,6 +1,7 @@
 """Small traversal set for compute-sanitizer (memcheck / racecheck / synccheck / initcheck).
 
-Usage: compute-sanitizer --tool <tool> python tools/sanitize_run.py [graph|hostloop]
+Usage: compute-sanitizer --tool <tool> python tests/sanitize_run.py [graph|hostloop]
+(lives under tests/ because it checks the results against the oracle)
   hostloop (default): every handle with ETG_HOST_LOOP (kernels launched from the host);
   graph: the shipping CUDA-graph conditional WHILE path (see tools/sanitize_graph_repro.cu
          for the tool's behaviour on conditional nodes without any library code).
@@ -12,6 +13,7 @@ import os
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
