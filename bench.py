@@ -530,6 +530,10 @@ def run_ours(args):
                                  f"launch of those same launches: {tr['alg_bytes_per_launch']:.0f} "
                                  f"(dram/algorithmic = {tr['dram_over_alg']:.2f})") if tr else None,
                 "peak_source": peak_src,
+                # SURVEY 8(d)'s pass criterion is the expand kernel's achieved DRAM GB/s: the
+                # ncu traffic of the same launches over their (serialised) durations
+                "dram_gbs_ncu": tr["dram_gbs_under_ncu"] if tr else None,
+                "dram_frac_ncu": tr["dram_gbs_under_ncu"] / peak if tr else None,
                 "algorithmic_bytes_per_launch": bytes_tot / max(1, launches_p),
                 "avg_launch_ms": exp_ms / max(1, launches_p),
                 "expand_share_of_call": exp_ms / max(1e-9, call_ms),
