@@ -241,6 +241,20 @@ void etg_free(etg_graph *g);
  * call), so only the first call pays the host-side setup.  Not re-entrant
  * across threads sharing one scratch buffer. */
 size_t etg_host_scratch_bytes(uint64_t n, uint64_t m, int has_weights, const etg_options *opt);
+/* Several traversals of ONE host graph (Proc. 1 per query; the paper times
+ * each with its own transfer, L247 -- here the CSR crosses the host link once
+ * for all of them): algs[q] / sources[q] for q < n_queries (sources ignored
+ * for CC), h_labels receives n_queries x n labels (query q at h_labels + q*n),
+ * st_or_null n_queries entries.  The weights are copied on an internal copy
+ * stream while the queries that need none run; each query's labels are
+ * copied back while the next one runs.  Same scratch, caching and error
+ * rules as etg_run_host (ETG_ENOWEIGHTS if a query needs weights and h_w is
+ * NULL). */
+etg_status etg_run_host_batch(uint64_t n, uint64_t m, const void *h_row_offsets, const uint32_t *h_col_idx,
+                              const uint32_t *h_weights, uint32_t n_queries, const int *algs,
+                              const uint32_t *sources, uint32_t *h_labels, void *d_scratch,
+                              size_t scratch_bytes, void *stream, const etg_options *opt,
+                              etg_stats *st_or_null);
 etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_row_offsets,
                         const uint32_t *h_col_idx, const uint32_t *h_weights,
                         uint32_t source, uint32_t *h_labels, void *d_scratch,

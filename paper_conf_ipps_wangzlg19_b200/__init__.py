@@ -22,7 +22,7 @@ import torch
 
 __all__ = [
     "EtgError", "Stats", "Graph", "load_csr", "csr_to_device", "to_u32_numpy",
-    "run_host", "host_scratch_bytes", "kernel_launches", "lib", "Comm",
+    "run_host", "run_host_batch", "host_scratch_bytes", "kernel_launches", "lib", "Comm",
     "SYMMETRIC", "NO_UDC", "NO_SMP", "OFFSETS_U64", "VALIDATE", "HOST_LOOP", "PROFILE", "SMP_SHARED",
     "HOST_EDGES", "PUSH",
     "INF", "CAP", "BFS", "SSSP", "CC", "SSWP",
@@ -86,6 +86,7 @@ def lib():
             "etg_free": (None, [p]),
             "etg_host_scratch_bytes": (sz, [u64, u64, ctypes.c_int, p]),
             "etg_run_host": (st, [ctypes.c_int, u64, u64, p, p, p, u32, p, p, sz, p, p, p]),
+            "etg_run_host_batch": (st, [u64, u64, p, p, p, u32, p, p, p, p, sz, p, p, p]),
             "etg_status_str": (ctypes.c_char_p, [st]),
             "etg_last_error": (ctypes.c_char_p, []),
             "etg_kernel_launches": (u64, []),
@@ -386,3 +387,32 @@ def run_host(alg: int, off: torch.Tensor, col: torch.Tensor, w: Optional[torch.T
                             _stream_ptr(stream), ctypes.byref(opt), ctypes.byref(st))
     _check(rc, "etg_run_host")
     return st
+
+
+def run_host_batch(queries, off: torch.Tensor, col: torch.Tensor, w: Optional[torch.Tensor],
+                   labels_out: torch.Tensor, scratch: torch.Tensor, *, K: int = 32, flags: int = 0,
+                   stream=None, sssp_delta: int = 0, symmetric: bool = False):
+    """Several traversals of one HOST graph, the CSR copied once:
+    ``queries`` = [(alg, source), ...]; ``labels_out`` a host int32 tensor of
+    len(queries) x n.  Returns the list of Stats."""
+    for t in (off, col, w, labels_out):
+        if t is not None and t.is_cuda:
+            raise EtgError("run_host_batch takes host tensors")
+    if off.dtype == torch.int64:
+        flags |= OFFSETS_U64
+    if symmetric:
+        flags |= SYMMETRIC
+    n = int(off.shape[0] - 1)
+    m = int(col.shape[0])
+    q = len(queries)
+    if labels_out.numel() < q * n or labels_out.dtype != torch.int32 or not labels_out.is_contiguous():
+        raise EtgError("labels_out must be a contiguous int32 host tensor of len(queries) x n")
+    algs = (ctypes.c_int * q)(*[a for a, _ in queries])
+    srcs = (ctypes.c_uint32 * q)(*[s for _, s in queries])
+    opt = Options(K, flags, _delta(sssp_delta))
+    sts = (Stats * q)()
+    rc = lib().etg_run_host_batch(n, m, _ptr(off), _ptr(col), _ptr(w), q, algs, srcs, _ptr(labels_out),
+                                  _ptr(scratch), scratch.numel() * scratch.element_size(),
+                                  _stream_ptr(stream), ctypes.byref(opt), sts)
+    _check(rc, "etg_run_host_batch")
+    return list(sts)

@@ -1207,17 +1207,30 @@ size_t etg_host_scratch_bytes(uint64_t n, uint64_t m, int has_weights, const etg
     o = align_up(o + (p.u64 ? 8 : 4) * (n + 1));
     o = align_up(o + 4 * m);
     if (has_weights) o = align_up(o + 4 * m);
-    o = align_up(o + 4 * n);
+    o = align_up(o + 4 * n);                 // two label buffers: the D2H of one query
+    o = align_up(o + 4 * n);                 // overlaps the traversal of the next
     return o + layout(n, m, p).total;
 }
 
-etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_off, const uint32_t *h_col,
-                        const uint32_t *h_w, uint32_t source, uint32_t *h_labels, void *d_scratch,
-                        size_t scratch_bytes, void *stream, const etg_options *opt, etg_stats *st) {
-    if (!h_off || (m && !h_col) || !h_labels || !d_scratch) return fail(ETG_EINVAL, "NULL argument");
-    if (alg < 0 || alg > 3) return fail(ETG_EINVAL, "alg must be 0..3");
+namespace {
+
+// Host-buffer entry (etg_run_host / etg_run_host_batch): H2D of the CSR into
+// the scratch, the queries on a handle over it, D2H of each query's labels.
+// Overlap: off and col go first on the call's stream; w follows on a copy
+// stream, so queries that need no weights (BFS, CC) run while it is in
+// flight; each query's labels go back on the copy stream while the next query
+// runs (two device label buffers).
+etg_status run_host_impl(uint64_t n, uint64_t m, const void *h_off, const uint32_t *h_col, const uint32_t *h_w,
+                         uint32_t nq, const int *algs, const uint32_t *sources, uint32_t *h_labels,
+                         void *d_scratch, size_t scratch_bytes, void *stream, const etg_options *opt,
+                         etg_stats *st) {
+    if (!h_off || (m && !h_col) || !h_labels || !d_scratch || !algs || (nq && !sources)) return fail(ETG_EINVAL, "NULL argument");
+    bool has_w = false;
+    for (uint32_t q = 0; q < nq; ++q) {
+        if (algs[q] < 0 || algs[q] > 3) return fail(ETG_EINVAL, "alg must be 0..3");
+        has_w |= (algs[q] == ALG_SSSP || algs[q] == ALG_SSWP);
+    }
     const Params p = derive(opt, env_tune());
-    const bool has_w = (alg == ALG_SSSP || alg == ALG_SSWP);
     if (has_w && !h_w) return fail(ETG_ENOWEIGHTS, "weights required");
     if (scratch_bytes < etg_host_scratch_bytes(n, m, has_w, opt)) return fail(ETG_ENOMEM, "scratch too small");
     cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -1233,16 +1246,17 @@ etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_off, cons
         d_w = reinterpret_cast<uint32_t *>(base + o);
         o = align_up(o + 4 * m);
     }
-    uint32_t *d_lab = reinterpret_cast<uint32_t *>(base + o);
+    uint32_t *d_lab[2];
+    d_lab[0] = reinterpret_cast<uint32_t *>(base + o);
     o = align_up(o + 4 * n);
-    ETG_CU(cudaMemcpyAsync(d_off, h_off, offsz, cudaMemcpyHostToDevice, s));
-    if (m) ETG_CU(cudaMemcpyAsync(d_col, h_col, 4 * m, cudaMemcpyHostToDevice, s));
-    if (has_w && m) ETG_CU(cudaMemcpyAsync(d_w, h_w, 4 * m, cudaMemcpyHostToDevice, s));
+    d_lab[1] = reinterpret_cast<uint32_t *>(base + o);
+    o = align_up(o + 4 * n);
     // A handle over this scratch layout is kept per thread and reused by the
     // next call with the same sizes, scratch, stream and options: the handle
     // holds only pointers into the scratch, so reuse just re-zeroes its
     // device control state; the host-side setup (pinned control block,
-    // events, the instantiated CUDA graph of the loop) is paid once.
+    // events, the instantiated CUDA graph of the loop, the copy stream) is
+    // paid once.
     struct Cached {
         uint64_t n, m;
         int has_w;
@@ -1251,19 +1265,42 @@ etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_off, cons
         cudaStream_t s;
         uint32_t K, flags, delta, tune;
         etg_graph *g;
+        cudaStream_t cs;         // copy stream (w in, labels out)
+        cudaEvent_t ev[5];       // w arrived; query done x 2; labels copied x 2
     };
     thread_local Cached cache[4] = {};
     thread_local unsigned next_slot = 0;
     const uint32_t K = opt ? opt->degree_limit_k : 0u, fl = opt ? opt->flags : 0u, dl = opt ? opt->sssp_delta : 0u;
     const uint32_t tune = env_tune();
-    etg_graph *g = nullptr;
+    Cached *cc = nullptr;
     for (Cached &c : cache)
         if (c.g && c.n == n && c.m == m && c.has_w == (int)has_w && c.scratch == d_scratch && c.bytes == scratch_bytes &&
             c.s == s && c.K == K && c.flags == fl && c.delta == dl && c.tune == tune) {
-            g = c.g;
+            cc = &c;
             break;
         }
     etg_status rc = ETG_OK;
+    if (!cc) {
+        Cached &c = cache[next_slot++ % 4];
+        if (c.g) {
+            etg_free(c.g);
+            cudaStreamDestroy(c.cs);
+            for (cudaEvent_t e : c.ev) cudaEventDestroy(e);
+            c.g = nullptr;
+        }
+        ETG_CU(cudaStreamCreateWithFlags(&c.cs, cudaStreamNonBlocking));
+        for (cudaEvent_t &e : c.ev) ETG_CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        c.n = n; c.m = m; c.has_w = (int)has_w; c.scratch = d_scratch; c.bytes = scratch_bytes; c.s = s;
+        c.K = K; c.flags = fl; c.delta = dl; c.tune = tune;
+        cc = &c;
+    }
+    cudaStream_t cs = cc->cs;
+    // H2D: offsets and columns on the call's stream; weights on the copy stream
+    ETG_CU(cudaMemcpyAsync(d_off, h_off, offsz, cudaMemcpyHostToDevice, s));
+    if (m) ETG_CU(cudaMemcpyAsync(d_col, h_col, 4 * m, cudaMemcpyHostToDevice, s));
+    if (has_w && m) ETG_CU(cudaMemcpyAsync(d_w, h_w, 4 * m, cudaMemcpyHostToDevice, cs));
+    ETG_CU(cudaEventRecord(cc->ev[0], cs));
+    etg_graph *g = cc->g;
     if (g) {
         ETG_CU(cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), s));
         ETG_CU(cudaMemsetAsync(g->ws + g->L.Q, 0, 4ull * g->L.nwords, s));
@@ -1276,17 +1313,44 @@ etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_off, cons
     } else {
         rc = etg_load_csr(&g, n, m, d_off, d_col, d_w, base + o, scratch_bytes - o, stream, opt, nullptr, 0, 0);
         if (rc != ETG_OK) return rc;
-        Cached &c = cache[next_slot++ % 4];
-        if (c.g) etg_free(c.g);
-        c = Cached{n, m, (int)has_w, d_scratch, scratch_bytes, s, K, fl, dl, tune, g};
+        cc->g = g;
     }
-    rc = run(g, alg, source, d_lab, st);
-    if (rc == ETG_OK) {
-        cudaError_t e = cudaMemcpyAsync(h_labels, d_lab, 4 * n, cudaMemcpyDeviceToHost, s);
-        if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-        if (e != cudaSuccess) rc = fail(ETG_ECUDA, std::string("run_host D2H: ") + cudaGetErrorString(e));
+    bool w_ready = !has_w;
+    for (uint32_t q = 0; q < nq && rc == ETG_OK; ++q) {
+        const int b = q & 1;
+        if (q >= 2) ETG_CU(cudaStreamWaitEvent(s, cc->ev[3 + b], 0));   // buffer b copied out
+        if (!w_ready && (algs[q] == ALG_SSSP || algs[q] == ALG_SSWP)) {
+            ETG_CU(cudaStreamWaitEvent(s, cc->ev[0], 0));
+            w_ready = true;
+        }
+        rc = run(g, algs[q], sources[q], d_lab[b], st ? st + q : nullptr);
+        if (rc != ETG_OK) break;
+        ETG_CU(cudaEventRecord(cc->ev[1 + b], s));
+        ETG_CU(cudaStreamWaitEvent(cs, cc->ev[1 + b], 0));
+        ETG_CU(cudaMemcpyAsync(h_labels + (size_t)q * n, d_lab[b], 4 * n, cudaMemcpyDeviceToHost, cs));
+        ETG_CU(cudaEventRecord(cc->ev[3 + b], cs));
     }
+    cudaError_t e = cudaStreamSynchronize(cs);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess && rc == ETG_OK) rc = fail(ETG_ECUDA, std::string("run_host D2H: ") + cudaGetErrorString(e));
     return rc;
+}
+
+}  // namespace
+
+etg_status etg_run_host(int alg, uint64_t n, uint64_t m, const void *h_off, const uint32_t *h_col,
+                        const uint32_t *h_w, uint32_t source, uint32_t *h_labels, void *d_scratch,
+                        size_t scratch_bytes, void *stream, const etg_options *opt, etg_stats *st) {
+    return run_host_impl(n, m, h_off, h_col, h_w, 1, &alg, &source, h_labels, d_scratch, scratch_bytes, stream,
+                         opt, st);
+}
+
+etg_status etg_run_host_batch(uint64_t n, uint64_t m, const void *h_off, const uint32_t *h_col,
+                              const uint32_t *h_w, uint32_t n_queries, const int *algs, const uint32_t *sources,
+                              uint32_t *h_labels, void *d_scratch, size_t scratch_bytes, void *stream,
+                              const etg_options *opt, etg_stats *st) {
+    return run_host_impl(n, m, h_off, h_col, h_w, n_queries, algs, sources, h_labels, d_scratch, scratch_bytes,
+                         stream, opt, st);
 }
 
 // ---- communicator ---------------------------------------------------------

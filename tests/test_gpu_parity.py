@@ -391,3 +391,28 @@ def test_sssp_delta_auto(c1):
     o1, c1_, w1 = g1.numpy()
     s = gg.first_source(c1)
     np.testing.assert_array_equal(U32(to_etg(g1, sssp_delta="auto").sssp(s)[0]), oracle.bfs(o1, c1_, s))
+
+
+def test_run_host_batch_matches(c1):
+    """Several queries on one host graph (the CSR crosses the link once; weights
+    arrive while BFS runs; labels go back while the next query runs)."""
+    off, col, w = c1.numpy()
+    o = torch.from_numpy(off.astype(np.int64)).to(torch.int32).pin_memory()
+    c = torch.from_numpy(col.view(np.int32)).pin_memory()
+    ww = torch.from_numpy(w.view(np.int32)).pin_memory()
+    srcs = gg.sample_sources(c1, 3, 11)
+    queries = [(etg.BFS, srcs[0]), (etg.SSSP, srcs[0]), (etg.SSWP, srcs[1]), (etg.BFS, srcs[2]),
+               (etg.SSSP, srcs[2])]
+    out = torch.empty(len(queries) * c1.n, dtype=torch.int32).pin_memory()
+    scratch = torch.empty(etg.host_scratch_bytes(c1.n, c1.m, True), dtype=torch.uint8, device="cuda")
+    for _ in range(2):                                   # the second call reuses the cached handle
+        out.fill_(7)
+        sts = etg.run_host_batch(queries, o, c, ww, out, scratch, sssp_delta="auto")
+        got = out.numpy().view(np.uint32).reshape(len(queries), c1.n)
+        fn = {etg.BFS: lambda s: oracle.bfs(off, col, s), etg.SSSP: lambda s: oracle.sssp(off, col, w, s),
+              etg.SSWP: lambda s: oracle.sswp(off, col, w, s)}
+        for k, (a, s) in enumerate(queries):
+            np.testing.assert_array_equal(got[k], fn[a](s), err_msg=f"query {k}")
+        assert len(sts) == len(queries) and all(st.iterations > 0 for st in sts)
+    with pytest.raises(etg.EtgError, match="ENOWEIGHTS"):
+        etg.run_host_batch(queries, o, c, None, out, scratch)
