@@ -178,6 +178,7 @@ struct etg_graph {
     uint64_t step_launches = 0;
     uint64_t step_acts = 0;               // activations counted so far (cumulative)
     bool delta_auto = false;              // sssp_delta was ETG_SSSP_DELTA_AUTO at load (sticky)
+    bool has_w = false;                   // weights given (or no edges)
     etg::Comm *comm = nullptr;            // communicator (borrowed), NULL = single partition
     bool push = false;                    // ETG_PUSH: source partition + fused push exchange
     uint32_t v_lo = 0, v_hi = 0;          // owned vertex range
@@ -756,7 +757,7 @@ etg_status run(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stat
 etg_status run_checked(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg_stats *st) {
     if (!g || !label) return fail(ETG_EINVAL, "null handle or label pointer");
     if (alg != ALG_CC && source >= g->n) return fail(ETG_EINVAL, "source >= n");
-    if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "graph loaded without weights");
+    if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->has_w) return fail(ETG_ENOWEIGHTS, "graph loaded without weights");
     if (alg == ALG_SSSP) {
         etg_status rc = resolve_delta(g);
         if (rc != ETG_OK) return rc;
@@ -1038,6 +1039,7 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
     g->off = d_row_offsets;
     g->col = d_col_idx;
     g->w = d_weights;
+    g->has_w = d_weights != nullptr || m == 0;   // no edge needs a weight (e.g. a partition that owns nothing)
     g->stream = static_cast<cudaStream_t>(stream);
     g->ws = static_cast<uint8_t *>(d_workspace);
     g->L = L;
@@ -1132,7 +1134,7 @@ etg_status etg_debug_expand_replay(etg_graph *g, int alg, uint32_t source, uint3
                                    uint64_t *edges, uint32_t *n_active) {
     if (!g || !d_label || !d_saved || !ms || !edges || !n_active) return fail(ETG_EINVAL, "NULL argument");
     if (alg < 0 || alg > 3) return fail(ETG_EINVAL, "alg must be 0..3");
-    if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "no weights");
+    if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->has_w) return fail(ETG_ENOWEIGHTS, "no weights");
     return g->p.u64 ? replay_impl<uint64_t>(g, alg, source, depth, tune, reps, d_label, d_saved, ms, edges, n_active)
                     : replay_impl<uint32_t>(g, alg, source, depth, tune, reps, d_label, d_saved, ms, edges, n_active);
 }
@@ -1141,7 +1143,7 @@ etg_status etg_step_begin(etg_graph *g, int alg, uint32_t source, uint32_t *d_la
     if (!g || !d_label || !n_active) return fail(ETG_EINVAL, "NULL argument");
     if (alg < 0 || alg > 3) return fail(ETG_EINVAL, "alg must be 0..3");
     if (alg != ALG_CC && source >= g->n) return fail(ETG_EINVAL, "source >= n");
-    if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->w) return fail(ETG_ENOWEIGHTS, "graph loaded without weights");
+    if ((alg == ALG_SSSP || alg == ALG_SSWP) && !g->has_w) return fail(ETG_ENOWEIGHTS, "graph loaded without weights");
     if (alg == ALG_CC && !(g->flags & ETG_SYMMETRIC)) return fail(ETG_ENOTSYM, "etg_cc needs ETG_SYMMETRIC");
     if (alg == ALG_SSSP && g->delta_auto)   // each rank would derive its own Delta from its own edges
         return fail(ETG_EINVAL, "step-wise runs need an explicit sssp_delta (every rank the same); "
@@ -1414,7 +1416,7 @@ uint64_t etg_kernel_launches(void) { return g_launches.load(); }
 
 etg_status etg_sssp_delta(etg_graph *g, uint32_t *delta) {
     if (!g || !delta) return fail(ETG_EINVAL, "NULL argument");
-    if (g->w) {
+    if (g->has_w) {
         etg_status rc = resolve_delta(g);
         if (rc != ETG_OK) return rc;
     }

@@ -174,3 +174,25 @@ def test_two_processes_cuda_ipc(exchange, tmp_path):
         g = graph_for(alg)
         got = np.concatenate([np.load(out + f".{alg}.{r}.npy") for r in range(2)])
         np.testing.assert_array_equal(got, expected(alg, g, gg.first_source(g)), err_msg=alg)
+
+
+@pytest.mark.parametrize("exchange", ["dest", "push"])
+def test_tiny_graphs_and_empty_ranges(exchange):
+    """Degenerate partitions: ranks whose owned range is empty (n < 32 P), a
+    graph smaller than one bitmap word, isolated vertices, and a source with no
+    out-edges -- every rank still agrees and the owned slices tile the result."""
+    edges = [(0, 1), (1, 2), (2, 0), (3, 4), (5, 5), (6, 7), (7, 6)]
+    for n, P in ((8, 2), (8, 4), (70, 4), (70, 3)):
+        g = gg.from_edges("tiny", n, [(u, v) for u, v in edges if u < n and v < n] + [(n - 2, n - 1)],
+                          weights=None, dedup=True)
+        g = gg.add_weights(g, 5)
+        for alg in (["sssp", "sswp"] if exchange == "push" else ["bfs", "sssp", "sswp"]):
+            for s in (0, 3, n - 1):                      # n - 1 has no out-edges
+                parts = parts_of(g, P, exchange=exchange)
+                labels, _ = edist.run_local(parts, ALG[alg], s)
+                np.testing.assert_array_equal(U32(labels), expected(alg, g, s), err_msg=f"{alg} n={n} P={P} s={s}")
+        gs = gg.symmetrize(g)
+        gs.w = None
+        parts = edist.local_partitions(gs.off, gs.col, None, gs.n, P, exchange=exchange, symmetric=True)
+        labels, _ = edist.run_local(parts, etg.CC, 0)
+        np.testing.assert_array_equal(U32(labels), expected("cc", gs, 0))
