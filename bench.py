@@ -605,7 +605,9 @@ def run_ours(args):
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": max_ms / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            # N > 1 partitions this same workload (strong scaling) unless --replicas
+            "scaling": "weak" if (args.replicas and world > 1) else "strong",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": config_desc(args.config) + "; " + "+".join(algs) + " per step",
                        "n": g.n, "m": g.m, "m_sym": m_sym, "K": args.K, "flags": args.flags,
                        "sssp_schedule": (f"wave, Delta={args.sssp_delta}" if str(args.sssp_delta) != "0"

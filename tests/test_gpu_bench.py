@@ -43,3 +43,11 @@ def test_bench_reference_arm():
     d = _run("--impl", "reference", "--config", "C1", "--steps", "2", "--warmup", "3")
     assert d["impl"] == "reference" and d["value"] > 0 and d["cpu_baseline"]["kind"] == "oracle"
     assert d["e2e"]["h2d_bytes_per_step"] == 0
+
+
+def test_bench_two_ranks_partitioned():
+    """--gpus 2 without torchrun: bench.py relaunches itself with two ranks
+    (here on one GPU), runs the partitioned path and rank 0 prints one line."""
+    d = _run("--gpus", "2", "--config", "C1", "--steps", "2", "--warmup", "3", "--sources", "4", "--no-e2e")
+    assert d["n_gpus"] == 2 and d["scaling"] == "strong" and d["value"] > 0
+    assert "partition" in d["config"]["parallelism"] and d["gpu_launches"] > 0
