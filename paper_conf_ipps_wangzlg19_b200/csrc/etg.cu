@@ -234,6 +234,18 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.filt_live = (g->tune & kTuneFiltLive) ? 1u
                   : (g->tune & kTuneFiltSnap) ? 0u
                   : (8ull * g->n > (uint64_t)g->l2_bytes ? 1u : 0u);
+    // own range: a push-partition rank activates only the vertices it owns (the
+    // only ones with local out-edges), so its init and scans cover [v_lo, v_hi)
+    // -- scan cost falls with P; the foreign labels it lowers (its proposal
+    // cache) are never re-scanned, so its pre-filter reads the live labels
+    const bool own = g->push && g->comm;
+    d.own_lo = own ? g->v_lo : 0u;
+    d.own_hi = own ? g->v_hi : (uint32_t)g->n;
+    d.own_w0 = d.own_lo >> 5;
+    d.own_w1 = own ? (uint32_t)((g->v_hi + 31ull) >> 5) : g->L.nwords;
+    if (d.own_w1 < d.own_w0) d.own_w1 = d.own_w0;
+    d.scan_t0 = d.own_w0 / (kScanV / 32);
+    if (own) d.filt_live = 1u;
     d.npeer = g->npeer;
     d.peer_rank = g->peer_rank;
     for (uint32_t k = 0; k <= kMaxPeer; ++k) d.peer_bounds[k] = g->peer_bounds[k];

@@ -131,6 +131,12 @@ struct Dev {
     uint32_t snap_used;         // SSSP/CC/SSWP, single GPU: a sole shadow stores the label it expands with
     uint32_t filt_live;         // SSSP/CC/SSWP pre-filter reads the live labels, not the snapshot (label +
                                 // snapshot larger than L2: one randomly gathered array instead of two)
+    // The vertex range this handle activates (a push-partition rank: its owned
+    // range, the only vertices with local out-edges; else [0, n)): init marks
+    // and the scan covers only these words, from scan tile scan_t0 on.
+    uint32_t own_lo, own_hi;    // vertices
+    uint32_t own_w0, own_w1;    // bitmap words [own_lo / 32, ceil(own_hi / 32))
+    uint32_t scan_t0;           // first scan tile (own_w0 / (kScanV / 32))
     // Fused push exchange (NEXT-3 over peer memory): a relaxation of a vertex
     // owned by rank q != peer_rank also lands, as a red.min/max, in rank q's
     // label array (device memory of another GPU reached over NVLink, or of
@@ -366,11 +372,11 @@ __global__ __launch_bounds__(kBlock) void init_kernel(Dev<OffT> d, uint32_t *lab
             d.V[k] = 0u;                                  // the first scan moves the source from Q to V
     }
     if (ALG == ALG_CC) {
-        for (uint32_t k = blockIdx.x * kBlock + threadIdx.x; k < d.nwords; k += stride) {
+        for (uint32_t k = d.own_w0 + blockIdx.x * kBlock + threadIdx.x; k < d.own_w1; k += stride) {
             const uint32_t lo = k * 32;
             d.Q[k] = lo >= n ? 0u : (n - lo >= 32 ? kFull : ((1u << (n - lo)) - 1u));
         }
-    } else if (blockIdx.x == 0 && threadIdx.x == 0) {
+    } else if (blockIdx.x == 0 && threadIdx.x == 0 && source >= d.own_lo && source < d.own_hi) {
         d.Q[source >> 5] = 1u << (source & 31);
     }
 }
@@ -450,7 +456,9 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
     Ctl *ctl = d.ctl;
     if (threadIdx.x == 0) s_acts = 0;
     const uint32_t epoch = cld<P>(ctl->epoch) & 0x3FFFFFFFu;
-    const uint32_t nscan = (d.n + kScanV - 1) / kScanV;
+    const uint32_t tile_words = kScanV / 32;
+    // tiles of the own range (at least one: its last tile publishes the sizes)
+    const uint32_t nscan = max(1u, (d.own_w1 + tile_words - 1) / tile_words - d.scan_t0);
     const uint32_t ts = d.ts, tsl = d.ts_log2;
     const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
     const uint32_t lt = (1u << lane) - 1u;
@@ -471,12 +479,16 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
         const uint32_t tile = (round == 0 && stat) ? blockIdx.x : s_tile;
         __syncthreads();                                  // all have read s_tile before it is reused
         if (tile >= nscan) break;
-        const uint32_t wbase = (tile * kWarps + warp) * kWPW;          // first word of this warp
+        const uint32_t wbase = ((tile + d.scan_t0) * kWarps + warp) * kWPW;   // first word of this warp
         // this warp's words: lane l holds words wbase + l + 32j (read, then cleared
-        // -- near-far SSSP keeps the deferred far bits)
+        // -- near-far SSSP keeps the deferred far bits); words outside the own
+        // range are not looked at
         uint32_t wq[kWPW / 32];
 #pragma unroll
-        for (int j = 0; j < kWPW / 32; ++j) wq[j] = xld<P>(&d.Q[wbase + 32 * j + lane]);
+        for (int j = 0; j < kWPW / 32; ++j) {
+            const uint32_t wd = wbase + 32 * j + lane;
+            wq[j] = (wd >= d.own_w0 && wd < d.own_w1) ? xld<P>(&d.Q[wd]) : 0u;
+        }
         uint32_t far_cnt = 0, far_min = kInf;
         const bool nf = d.nf_delta != 0;
 #pragma unroll
@@ -507,10 +519,11 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                     uint32_t lv[2 * kG], sv[2 * kG];
 #pragma unroll
                     for (int r = 0; r < 2 * kG; ++r) {
-                        const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
+                        const uint32_t wd = wbase + 32 * j + k0 + r;
+                        const uint32_t v = wd * 32 + lane;
                         lv[r] = 0;
                         sv[r] = 0;
-                        if (v < d.n) {
+                        if (v < d.n && wd >= d.own_w0 && wd < d.own_w1) {
                             lv[r] = __ldcg(&label[v]);
                             sv[r] = __ldcg(&d.snap[v]);
                         }
