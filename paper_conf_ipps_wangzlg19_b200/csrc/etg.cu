@@ -120,7 +120,7 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
     };
     const uint64_t max_shadows = p.udc ? (m + p.K - 1) / p.K + n : n;   // sum ceil(d/K) <= m/K + |F|
     const uint64_t max_tiles = (max_shadows + 31) / 32 + 2;      // sized for the smallest tile (32)
-    const uint64_t max_scan_tiles = (n + kScanV - 1) / kScanV + 2;
+    const uint64_t max_scan_tiles = (n + 1023) / 1024 + 2;      // sized for the smallest scan tile (4 rows per warp)
     const uint64_t words = (n + 31) / 32;
     const uint64_t tile_words = kScanV / 32;
     L.nwords = (uint32_t)((words + tile_words - 1) / tile_words * tile_words);
@@ -162,6 +162,7 @@ struct etg_graph {
     int l2_bytes = 0;
     uint32_t tune = 0;                    // ETG_TUNE (experiments only)
     int grid_scan = 0;
+    int scan_kw = kWPW;                   // bitmap words per scan warp (tile = 8 x scan_kw x 32 vertices)
     int grid_init = 0;
     Ctl *h_ctl = nullptr;                 // pinned host mirror for readback
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
@@ -244,7 +245,7 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.own_w0 = d.own_lo >> 5;
     d.own_w1 = own ? (uint32_t)((g->v_hi + 31ull) >> 5) : g->L.nwords;
     if (d.own_w1 < d.own_w0) d.own_w1 = d.own_w0;
-    d.scan_t0 = d.own_w0 / (kScanV / 32);
+    d.scan_t0 = d.own_w0 / ((uint32_t)kWarps * (uint32_t)g->scan_kw);
     if (own) d.filt_live = 1u;
     d.npeer = g->npeer;
     d.peer_rank = g->peer_rank;
@@ -332,11 +333,22 @@ const void *init_fn(int alg) {
     }
 }
 
-template <class OffT>
-const void *scan_fn(bool udc, int alg) {
+template <class OffT, int KW>
+const void *scan_fn_kw(bool udc, int alg) {
     if (alg == ALG_BFS)
-        return udc ? (const void *)udc_scan_kernel<OffT, true, true> : (const void *)udc_scan_kernel<OffT, false, true>;
-    return udc ? (const void *)udc_scan_kernel<OffT, true, false> : (const void *)udc_scan_kernel<OffT, false, false>;
+        return udc ? (const void *)udc_scan_kernel<OffT, true, true, KW> : (const void *)udc_scan_kernel<OffT, false, true, KW>;
+    return udc ? (const void *)udc_scan_kernel<OffT, true, false, KW> : (const void *)udc_scan_kernel<OffT, false, false, KW>;
+}
+
+// the scan kernel of a handle: KW = g->scan_kw bitmap words (rows) per warp
+template <class OffT>
+const void *scan_fn(const etg_graph *g, int alg) {
+    switch (g->scan_kw) {
+        case 4: return scan_fn_kw<OffT, 4>(g->p.udc, alg);
+        case 8: return scan_fn_kw<OffT, 8>(g->p.udc, alg);
+        case 16: return scan_fn_kw<OffT, 16>(g->p.udc, alg);
+        default: return scan_fn_kw<OffT, kWPW>(g->p.udc, alg);
+    }
 }
 
 // second argument of the expand kernels: CTA kernel -> staging capacity in
@@ -409,7 +421,7 @@ etg_status build_graph(etg_graph *g, int alg) {
     int use_cond = 1;
     void *scan_args[] = {&d, &cond, &use_cond};
     memset(&kp, 0, sizeof(kp));
-    kp.func = const_cast<void *>(scan_fn<OffT>(g->p.udc, alg));
+    kp.func = const_cast<void *>(scan_fn<OffT>(g, alg));
     kp.gridDim = dim3(g->grid_scan);
     kp.blockDim = dim3(kBlock);
     kp.kernelParams = scan_args;
@@ -450,7 +462,7 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
     int zero = 0;
     void *scan_args[] = {&d, &none, &zero};
     // A2 of the initial active set (Proc. 1 "Init actSet")
-    ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+    ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
     uint64_t launches = 2;                       // init (+ control block), first scan
     if (persist) {
         // the whole loop in one cooperative launch (all CTAs co-resident)
@@ -473,7 +485,7 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
             if (profile) ETG_CU(cudaEventRecord(g->pev[0], s));
             ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
             if (profile) ETG_CU(cudaEventRecord(g->pev[1], s));
-            ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+            ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
             if (profile) ETG_CU(cudaEventRecord(g->pev[2], s));
             launches += 2;
             if (profile) {
@@ -558,7 +570,7 @@ etg_status step_scan_impl(etg_graph *g, uint32_t *n_active) {
             ctl_rescan_kernel<<<1, 1, 0, s>>>(g->ctl);
             g->step_launches += 1;
         }
-        ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, g->step_alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+        ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, g->step_alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
         g->step_launches += 1;
         ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
         ETG_CU(cudaStreamSynchronize(s));
@@ -818,7 +830,12 @@ etg_status udc_impl(etg_graph *g, const uint32_t *act, uint32_t n_act, uint32_t 
     cudaStream_t s = g->stream;
     ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, nullptr, 0);
     if (n_act) mark_kernel<<<g->num_sms, kBlock, 0, s>>>(d.Q, act, n_act);
-    udc_scan_kernel<OffT, true, false><<<g->grid_scan, kBlock, 0, s>>>(d, 0, 0);
+    {
+        cudaGraphConditionalHandle none = 0;
+        int zero = 0;
+        void *args[] = {&d, &none, &zero};
+        ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, ALG_SSSP), dim3(g->grid_scan), dim3(kBlock), args, 0, s));
+    }
     ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     ETG_CU(cudaStreamSynchronize(s));
     *n_out = g->h_ctl->nshadow;
@@ -850,13 +867,13 @@ etg_status replay_impl(etg_graph *g, int alg, uint32_t source, uint32_t depth, u
     ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, label, source);
     void *iargs[] = {&d, &label, &source};
     ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), iargs, 0, s));
-    ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+    ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
     for (;;) {
         ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
         ETG_CU(cudaStreamSynchronize(s));
         if (g->h_ctl->depth >= depth || g->h_ctl->nF == 0) break;
         ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
-        ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g->p.udc, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+        ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
     }
     ETG_CU(cudaMemsetAsync(&g->ctl->reached_v, 0, 8, s));
     ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
@@ -1089,7 +1106,20 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
     g->tune = tune;
     // no more scan CTAs than scan tiles, no more init CTAs than 256-vertex
     // blocks: a small graph does not launch hundreds of CTAs that exit at once
-    const uint64_t nscan = (n + kScanV - 1) / kScanV, ninit = (std::max<uint64_t>(n, L.nwords) + kBlock - 1) / kBlock;
+    // scan tiles: 32 rows per warp (8,192-vertex tiles) when that still gives
+    // >= 2 tiles per SM, else fewer rows per warp -- a small graph's scan is
+    // then short dependent chains on many SMs; ETG_SCAN_KW (4, 8, 16, 32)
+    // overrides for experiments
+    int kw = kWPW;
+    while (kw > 4 && (n + 256ull * kw - 1) / (256ull * kw) < 2ull * (uint64_t)g->num_sms) kw >>= 1;
+    if (const char *e_kw = getenv("ETG_SCAN_KW")) {
+        const int v = atoi(e_kw);
+        if (v == 4 || v == 8 || v == 16 || v == 32) kw = v;
+    }
+    if (p.persist) kw = kWPW;             // the persistent loop's scan phase uses 32 rows
+    g->scan_kw = kw;
+    const uint64_t nscan = (n + 256ull * kw - 1) / (256ull * kw);
+    const uint64_t ninit = (std::max<uint64_t>(n, L.nwords) + kBlock - 1) / kBlock;
     g->grid_scan = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)g->num_sms * 4, nscan));
     g->grid_init = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)g->num_sms * 8, ninit));
     if (flags & ETG_VALIDATE) {

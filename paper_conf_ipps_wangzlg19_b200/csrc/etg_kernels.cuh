@@ -446,17 +446,23 @@ __device__ __forceinline__ void lookback_resolve(const unsigned long long (&r)[N
     else p -= 32 * N;
 }
 
-template <class OffT, bool UDC, bool BFSLAB, bool P>
+// KW = bitmap words (rows of 32 vertices) per warp: a scan tile covers
+// kWarps * KW * 32 vertices.  A warp walks its rows one after another, so KW is
+// the length of its dependent chain: large graphs use KW = 32 (8,192-vertex
+// tiles, fewest tiles and look-back steps), small ones fewer rows per warp,
+// so their scans are short chains on many SMs instead of long ones on few.
+template <class OffT, bool UDC, bool BFSLAB, bool P, int KW = kWPW>
 __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditionalHandle cond, int use_cond) {
     typedef unsigned long long u64;
     __shared__ uint32_t s_tile;
     __shared__ u64 s_prefix;
     __shared__ u64 s_wsum[kWarps];
+    static_assert(KW >= 4 && KW <= 32 && (32 % KW) == 0, "rows per warp");
     __shared__ uint32_t s_acts;                           // activations of this CTA (one global atomic)
     Ctl *ctl = d.ctl;
     if (threadIdx.x == 0) s_acts = 0;
     const uint32_t epoch = cld<P>(ctl->epoch) & 0x3FFFFFFFu;
-    const uint32_t tile_words = kScanV / 32;
+    const uint32_t tile_words = (uint32_t)kWarps * KW;
     // tiles of the own range (at least one: its last tile publishes the sizes)
     const uint32_t nscan = max(1u, (d.own_w1 + tile_words - 1) / tile_words - d.scan_t0);
     const uint32_t ts = d.ts, tsl = d.ts_log2;
@@ -479,20 +485,19 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
         const uint32_t tile = (round == 0 && stat) ? blockIdx.x : s_tile;
         __syncthreads();                                  // all have read s_tile before it is reused
         if (tile >= nscan) break;
-        const uint32_t wbase = ((tile + d.scan_t0) * kWarps + warp) * kWPW;   // first word of this warp
+        const uint32_t wbase = ((tile + d.scan_t0) * kWarps + warp) * KW;   // first word of this warp
         // this warp's words: lane l holds words wbase + l + 32j (read, then cleared
         // -- near-far SSSP keeps the deferred far bits); words outside the own
         // range are not looked at
-        uint32_t wq[kWPW / 32];
-#pragma unroll
-        for (int j = 0; j < kWPW / 32; ++j) {
-            const uint32_t wd = wbase + 32 * j + lane;
-            wq[j] = (wd >= d.own_w0 && wd < d.own_w1) ? xld<P>(&d.Q[wd]) : 0u;
+        uint32_t wq[1];
+        {
+            const uint32_t wd = wbase + lane;
+            wq[0] = (lane < (uint32_t)KW && wd >= d.own_w0 && wd < d.own_w1) ? xld<P>(&d.Q[wd]) : 0u;
         }
         uint32_t far_cnt = 0, far_min = kInf;
         const bool nf = d.nf_delta != 0;
 #pragma unroll
-        for (int j = 0; j < kWPW / 32; ++j)
+        for (int j = 0; j < 1; ++j)
             if (wq[j]) {
                 d.Q[wbase + 32 * j + lane] = 0u;
                 if (BFSLAB) {
@@ -513,9 +518,9 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
             // -- its snapshot is not refreshed, so it stays "moved" and is
             // looked at again by every later scan until the threshold passes it.
 #pragma unroll
-            for (int j = 0; j < kWPW / 32; ++j) {
+            for (int j = 0; j < 1; ++j) {
                 uint32_t mine = 0;
-                for (uint32_t k0 = 0; k0 < 32; k0 += 2 * kG) {
+                for (uint32_t k0 = 0; k0 < (uint32_t)KW; k0 += 2 * kG) {
                     uint32_t lv[2 * kG], sv[2 * kG];
 #pragma unroll
                     for (int r = 0; r < 2 * kG; ++r) {
@@ -523,7 +528,7 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                         const uint32_t v = wd * 32 + lane;
                         lv[r] = 0;
                         sv[r] = 0;
-                        if (v < d.n && wd >= d.own_w0 && wd < d.own_w1) {
+                        if (k0 + r < (uint32_t)KW && v < d.n && wd >= d.own_w0 && wd < d.own_w1) {
                             lv[r] = __ldcg(&label[v]);
                             sv[r] = __ldcg(&d.snap[v]);
                         }
@@ -558,8 +563,8 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
         u64 wsum = 0;
         uint32_t nbits = 0;
 #pragma unroll
-        for (int j = 0; j < kWPW / 32; ++j) {
-            for (uint32_t k0 = 0; k0 < 32; k0 += kG) {
+        for (int j = 0; j < 1; ++j) {
+            for (uint32_t k0 = 0; k0 < (uint32_t)KW; k0 += kG) {
                 uint32_t word[kG], any = 0;
 #pragma unroll
                 for (int r = 0; r < kG; ++r) {
@@ -643,8 +648,8 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
         // pass 2: write the compacted entries, in vertex order, coalesced
         u64 run = s_prefix + wprefix;
 #pragma unroll
-        for (int j = 0; j < kWPW / 32; ++j) {
-            for (uint32_t k0 = 0; k0 < 32; k0 += kG) {
+        for (int j = 0; j < 1; ++j) {
+            for (uint32_t k0 = 0; k0 < (uint32_t)KW; k0 += kG) {
                 uint32_t word[kG], any = 0;
 #pragma unroll
                 for (int r = 0; r < kG; ++r) {
@@ -724,10 +729,10 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
     if (threadIdx.x == 0 && s_acts) atomicAdd(&ctl->activations, (u64)s_acts);   // result unused: RED
 }
 
-template <class OffT, bool UDC, bool BFSLAB>
+template <class OffT, bool UDC, bool BFSLAB, int KW = kWPW>
 __global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGraphConditionalHandle cond,
                                                           int use_cond) {
-    scan_phase<OffT, UDC, BFSLAB, false>(d, cond, use_cond);
+    scan_phase<OffT, UDC, BFSLAB, false, KW>(d, cond, use_cond);
 }
 
 // ------------------------------------------------------------------------- //
