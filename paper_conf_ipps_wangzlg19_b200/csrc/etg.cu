@@ -482,11 +482,13 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
             ETG_CU(cudaMemcpyAsync(&g->h_ctl->more, &g->ctl->more, 4, cudaMemcpyDeviceToHost, s));
             ETG_CU(cudaStreamSynchronize(s));
             if (g->h_ctl->more == 0) break;
+            nvtxRangePushA("etg_iteration");
             if (profile) ETG_CU(cudaEventRecord(g->pev[0], s));
             ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
             if (profile) ETG_CU(cudaEventRecord(g->pev[1], s));
             ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
             if (profile) ETG_CU(cudaEventRecord(g->pev[2], s));
+            nvtxRangePop();
             launches += 2;
             if (profile) {
                 ETG_CU(cudaEventSynchronize(g->pev[2]));
@@ -710,6 +712,7 @@ etg_status comm_run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *out, 
     rc = live_count(live);
     if (rc != ETG_OK) return rc;
     while (live) {
+        nvtxRangePushA("etg_iteration");
         rc = step_expand_impl<OffT>(g);
         if (rc != ETG_OK) return rc;
         if (!g->push && multi) {
@@ -723,6 +726,7 @@ etg_status comm_run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *out, 
         rc = step_scan_impl<OffT>(g, &nact);
         if (rc != ETG_OK) return rc;
         rc = live_count(live);           // also: nobody writes iteration k+1 into a copy still being scanned
+        nvtxRangePop();
         if (rc != ETG_OK) return rc;
     }
     ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));

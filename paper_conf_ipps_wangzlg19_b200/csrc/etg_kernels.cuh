@@ -1359,15 +1359,15 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
                 my_passes += x;
                 return;
             }
-            if (PEER && ALG != ALG_BFS) {
+            if constexpr (PEER && ALG != ALG_BFS) {
 #pragma unroll
                 for (int r = 0; r < kRB; ++r)
                     if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) commit_peer<OffT, ALG>(d, label, u[r], c[r], keep);
-                return;
-            }
+            } else {
 #pragma unroll
-            for (int r = 0; r < kRB; ++r)
-                if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, markQ);
+                for (int r = 0; r < kRB; ++r)
+                    if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, markQ);
+            }
         };
         stage_a(u0, c0, am0);
         if (!d.ahead) {
