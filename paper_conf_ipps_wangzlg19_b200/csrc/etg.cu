@@ -690,28 +690,34 @@ etg_status comm_run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *out, 
     etg_status rc = step_begin_impl<OffT>(g, alg, source, lab, &nact, 0);
     if (rc != ETG_OK) return rc;
     ETG_BAR(c, "init");                  // every copy initialised before anyone writes into it
+    uint64_t nf_all = 0;                 // compacted frontier summed over the ranks (statistics)
     auto live_count = [&](uint64_t &live) -> etg_status {
         // push: any rank with work (compacted vertices or deferred far ones);
         // destination: the activation count, identical on every rank
-        uint64_t mine = g->push ? (uint64_t)g->h_ctl->more : (uint64_t)nact;
+        uint64_t mine[2] = {g->push ? (uint64_t)g->h_ctl->more : (uint64_t)nact, (uint64_t)g->h_ctl->nF};
         if (!multi) {
-            live = mine;
+            live = mine[0];
+            nf_all = mine[1];
             return ETG_OK;
         }
-        etg_status r = comm_gather(c, 0, &mine, 1, all);
+        etg_status r = comm_gather(c, 6, mine, 2, all);   // positions 6, 7
         if (r != ETG_OK) return r;
         live = 0;
+        nf_all = 0;
         for (int q = 0; q < c.world; ++q) {
-            if (!g->push && all[q][0] != mine)
+            if (!g->push && all[q][6] != mine[0])
                 return fail(ETG_ENCCL, "ranks disagree on the active-set size (not the same graph or arguments?)");
-            live += all[q][0];
+            live += all[q][6];
+            nf_all += all[q][7];
         }
         return ETG_OK;
     };
     uint64_t live = 0;
     rc = live_count(live);
     if (rc != ETG_OK) return rc;
+    uint32_t trips = 0;                  // Proc. 1 iterations: trips that expand a non-empty frontier
     while (live) {
+        if (nf_all) ++trips;             // (on some rank: the same count on every rank)
         nvtxRangePushA("etg_iteration");
         rc = step_expand_impl<OffT>(g);
         if (rc != ETG_OK) return rc;
@@ -758,7 +764,7 @@ etg_status comm_run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *out, 
     }
     if (st) {
         memset(st, 0, sizeof(*st));
-        st->iterations = h.iterations;
+        st->iterations = trips;          // global (a rank's own non-empty frontiers can be fewer)
         st->edges_processed = tot[0];
         st->shadows = tot[1];
         st->frontier_total = tot[2];

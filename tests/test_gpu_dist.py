@@ -196,3 +196,16 @@ def test_tiny_graphs_and_empty_ranges(exchange):
         parts = edist.local_partitions(gs.off, gs.col, None, gs.n, P, exchange=exchange, symmetric=True)
         labels, _ = edist.run_local(parts, etg.CC, 0)
         np.testing.assert_array_equal(U32(labels), expected("cc", gs, 0))
+
+
+def test_loop_trips_are_global():
+    """etg_stats.iterations of a communicator handle counts the loop trips, the
+    same on every rank: BFS along a directed path of L vertices takes L - 1."""
+    L = 200
+    off = torch.zeros(L + 1, dtype=torch.int64)
+    off[1:L] = torch.arange(1, L)
+    off[L:] = L - 1
+    col = torch.arange(1, L, dtype=torch.int64)
+    parts = edist.local_partitions(off, col, None, L, 3)
+    sts = edist._in_threads([lambda p=p: p.run(etg.BFS, 0)[1].iterations for p in parts])
+    assert sts == [L - 1] * 3
