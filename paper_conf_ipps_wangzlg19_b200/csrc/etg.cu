@@ -163,6 +163,11 @@ struct etg_graph {
     uint32_t tune = 0;                    // ETG_TUNE (experiments only)
     int grid_scan = 0;
     int scan_kw = kWPW;                   // bitmap words per scan warp (tile = 8 x scan_kw x 32 vertices)
+    uint32_t scan_smem = 0;               // scan: dynamic shared memory (offset staging buffers + mbarriers)
+    uint32_t scan_rows = 0;               // scan: active rows from which a warp stages its offsets (0: never)
+    uint32_t split = 8;                   // expand: max warps sharing one tile in sparse iterations (ETG_SPLIT)
+    bool pdl = false;                     // loop graph: programmatic expand -> scan edges (ETG_PDL=1; measured
+                                          // 1 % slower on C2, per-iteration floor unchanged: off by default)
     int grid_init = 0;
     Ctl *h_ctl = nullptr;                 // pinned host mirror for readback
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
@@ -247,6 +252,8 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     if (d.own_w1 < d.own_w0) d.own_w1 = d.own_w0;
     d.scan_t0 = d.own_w0 / ((uint32_t)kWarps * (uint32_t)g->scan_kw);
     if (own) d.filt_live = 1u;
+    d.scan_rows = g->scan_smem ? g->scan_rows : 0u;
+    d.split = g->split;
     d.npeer = g->npeer;
     d.peer_rank = g->peer_rank;
     for (uint32_t k = 0; k <= kMaxPeer; ++k) d.peer_bounds[k] = g->peer_bounds[k];
@@ -351,6 +358,19 @@ const void *scan_fn(const etg_graph *g, int alg) {
     }
 }
 
+// one scan launch on stream s (the handle's grid and shared memory)
+template <class OffT>
+cudaError_t launch_scan(const etg_graph *g, int alg, void **args, cudaStream_t s) {
+    return cudaLaunchKernel(scan_fn<OffT>(g, alg), dim3(g->grid_scan), dim3(kBlock), args, g->scan_smem, s);
+}
+
+// shared memory of the scan kernels with KW rows per warp: per warp KW * 32 + 1
+// offsets rounded up to 16 bytes, plus one mbarrier
+template <class OffT>
+uint32_t scan_smem_bytes(int kw) {
+    return (uint32_t)(kWarps * ((uint32_t)kw * 32u + 16u / (uint32_t)sizeof(OffT)) * sizeof(OffT) + kWarps * 8);
+}
+
 // second argument of the expand kernels: CTA kernel -> staging capacity in
 // edges; warp kernel -> words per SMP stage array
 uint32_t expand_arg(const Params &p) { return p.warp ? 32u * (p.K + 6u) : p.ts * p.K; }
@@ -420,14 +440,31 @@ etg_status build_graph(etg_graph *g, int alg) {
 
     int use_cond = 1;
     void *scan_args[] = {&d, &cond, &use_cond};
-    memset(&kp, 0, sizeof(kp));
-    kp.func = const_cast<void *>(scan_fn<OffT>(g, alg));
-    kp.gridDim = dim3(g->grid_scan);
-    kp.blockDim = dim3(kBlock);
-    kp.kernelParams = scan_args;
-    ETG_CU(cudaGraphAddKernelNode(&n_scan, body, &n_exp, 1, &kp));
+    // expand -> scan: a programmatic edge (PDL, ETG_PDL=0 disables) -- the
+    // scan grid launches while the expand drains and waits on the device
+    cudaGraphNodeParams np = {};
+    np.type = cudaGraphNodeTypeKernel;
+    np.kernel.func = const_cast<void *>(scan_fn<OffT>(g, alg));
+    np.kernel.gridDim = dim3(g->grid_scan);
+    np.kernel.blockDim = dim3(kBlock);
+    np.kernel.sharedMemBytes = g->scan_smem;
+    np.kernel.kernelParams = scan_args;
+    cudaGraphEdgeData ed = {};
+    if (g->pdl) {
+        ed.from_port = cudaGraphKernelNodePortProgrammatic;
+        ed.type = cudaGraphDependencyTypeProgrammatic;
+    }
+    ETG_CU(cudaGraphAddNode_v2(&n_scan, body, &n_exp, &ed, 1, &np));
 
-    ETG_CU(cudaGraphInstantiate(&g->exec[alg], graph, 0));
+    cudaError_t ie = cudaGraphInstantiate(&g->exec[alg], graph, 0);
+    if (ie != cudaSuccess && g->pdl) {
+        // programmatic edges not accepted here: plain edges
+        (void)cudaGetLastError();
+        cudaGraphDestroy(graph);
+        g->pdl = false;
+        return build_graph<OffT>(g, alg);
+    }
+    ETG_CU(ie);
     g->graph[alg] = graph;
     return ETG_OK;
 }
@@ -462,7 +499,7 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
     int zero = 0;
     void *scan_args[] = {&d, &none, &zero};
     // A2 of the initial active set (Proc. 1 "Init actSet")
-    ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+    ETG_CU(launch_scan<OffT>(g, alg, scan_args, s));
     uint64_t launches = 2;                       // init (+ control block), first scan
     if (persist) {
         // the whole loop in one cooperative launch (all CTAs co-resident)
@@ -486,7 +523,7 @@ etg_status run_impl(etg_graph *g, int alg, uint32_t source, uint32_t *label, etg
             if (profile) ETG_CU(cudaEventRecord(g->pev[0], s));
             ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
             if (profile) ETG_CU(cudaEventRecord(g->pev[1], s));
-            ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+            ETG_CU(launch_scan<OffT>(g, alg, scan_args, s));
             if (profile) ETG_CU(cudaEventRecord(g->pev[2], s));
             nvtxRangePop();
             launches += 2;
@@ -572,7 +609,7 @@ etg_status step_scan_impl(etg_graph *g, uint32_t *n_active) {
             ctl_rescan_kernel<<<1, 1, 0, s>>>(g->ctl);
             g->step_launches += 1;
         }
-        ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, g->step_alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+        ETG_CU(launch_scan<OffT>(g, g->step_alg, scan_args, s));
         g->step_launches += 1;
         ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
         ETG_CU(cudaStreamSynchronize(s));
@@ -844,7 +881,7 @@ etg_status udc_impl(etg_graph *g, const uint32_t *act, uint32_t n_act, uint32_t 
         cudaGraphConditionalHandle none = 0;
         int zero = 0;
         void *args[] = {&d, &none, &zero};
-        ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, ALG_SSSP), dim3(g->grid_scan), dim3(kBlock), args, 0, s));
+        ETG_CU(launch_scan<OffT>(g, ALG_SSSP, args, s));
     }
     ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     ETG_CU(cudaStreamSynchronize(s));
@@ -877,13 +914,13 @@ etg_status replay_impl(etg_graph *g, int alg, uint32_t source, uint32_t depth, u
     ctl_begin_kernel<<<1, 1, 0, s>>>(g->ctl, label, source);
     void *iargs[] = {&d, &label, &source};
     ETG_CU(cudaLaunchKernel(init_fn<OffT>(alg), dim3(g->grid_init), dim3(kBlock), iargs, 0, s));
-    ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+    ETG_CU(launch_scan<OffT>(g, alg, scan_args, s));
     for (;;) {
         ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
         ETG_CU(cudaStreamSynchronize(s));
         if (g->h_ctl->depth >= depth || g->h_ctl->nF == 0) break;
         ETG_CU(cudaLaunchKernel(ex.fn, ex.grid, dim3(kBlock), exp_args, ex.smem, s));
-        ETG_CU(cudaLaunchKernel(scan_fn<OffT>(g, alg), dim3(g->grid_scan), dim3(kBlock), scan_args, 0, s));
+        ETG_CU(launch_scan<OffT>(g, alg, scan_args, s));
     }
     ETG_CU(cudaMemsetAsync(&g->ctl->reached_v, 0, 8, s));
     ETG_CU(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
@@ -1130,7 +1167,28 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
     g->scan_kw = kw;
     const uint64_t nscan = (n + 256ull * kw - 1) / (256ull * kw);
     const uint64_t ninit = (std::max<uint64_t>(n, L.nwords) + kBlock - 1) / kBlock;
-    g->grid_scan = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)g->num_sms * 4, nscan));
+    // scan offset staging (a 16-byte-aligned offset array; not in the persistent
+    // loop): a warp with >= ETG_SCAN_ROWS active rows (default 4; 0 disables)
+    // bulk-copies its offsets into shared memory
+    if (const char *e_s = getenv("ETG_SPLIT")) g->split = (uint32_t)std::max(1, atoi(e_s));
+    if (const char *e_p = getenv("ETG_PDL")) g->pdl = atoi(e_p) != 0;
+    g->scan_rows = 4;
+    if (const char *e_r = getenv("ETG_SCAN_ROWS")) g->scan_rows = (uint32_t)atoi(e_r);
+    g->scan_smem = 0;
+    int scan_occ = 4;
+    if (g->scan_rows && (reinterpret_cast<uintptr_t>(d_row_offsets) & 15u) == 0 && !p.persist) {
+        g->scan_smem = p.u64 ? scan_smem_bytes<uint64_t>(kw) : scan_smem_bytes<uint32_t>(kw);
+        for (int a = 0; a < 2; ++a) {
+            const int alg = a ? ALG_SSSP : ALG_BFS;
+            const void *fn = p.u64 ? scan_fn<uint64_t>(g, alg) : scan_fn<uint32_t>(g, alg);
+            int nb = 0;
+            if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->scan_smem)) != cudaSuccess ||
+                (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, kBlock, g->scan_smem)) != cudaSuccess)
+                return bail(fail(ETG_ECUDA, std::string("load (scan): ") + cudaGetErrorString(e)));
+            scan_occ = std::max(1, std::min(scan_occ, nb));
+        }
+    }
+    g->grid_scan = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)g->num_sms * scan_occ, nscan));
     g->grid_init = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)g->num_sms * 8, ninit));
     if (flags & ETG_VALIDATE) {
         etg_status s = p.u64 ? validate_impl<uint64_t>(g) : validate_impl<uint32_t>(g);

@@ -131,6 +131,9 @@ struct Dev {
     uint32_t snap_used;         // SSSP/CC/SSWP, single GPU: a sole shadow stores the label it expands with
     uint32_t filt_live;         // SSSP/CC/SSWP pre-filter reads the live labels, not the snapshot (label +
                                 // snapshot larger than L2: one randomly gathered array instead of two)
+    uint32_t split;             // expand: max warps sharing one tile in sparse iterations (1: no split)
+    uint32_t scan_rows;         // scan: a warp with >= scan_rows active rows stages its offsets in shared
+                                // memory with one bulk copy (0: never; needs the dynamic shared memory)
     // The vertex range this handle activates (a push-partition rank: its owned
     // range, the only vertices with local out-edges; else [0, n)): init marks
     // and the scan covers only these words, from scan tile scan_t0 on.
@@ -311,6 +314,38 @@ __device__ __forceinline__ uint32_t udc_count(D deg, uint32_t K, uint32_t klog) 
     return (uint32_t)((deg - 1) / (D)K + 1);
 }
 
+// ---- mbarrier / bulk-copy helpers (SMP stages, scan offset staging) ----
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
+    asm volatile("{\n .reg .pred p;\n WAIT_%=:\n"
+                 " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+                 " @!p bra WAIT_%=;\n}" :: "r"(smem_u32(b)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+// TMA bulk copy global -> shared (16-byte aligned, size multiple of 16), completing on mbarrier b
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *b, uint64_t pol) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+                 :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(b)), "l"(pol) : "memory");
+}
+// ... without an L2 cache hint
+__device__ __forceinline__ void bulk_g2s_plain(void *dst, const void *src, uint32_t bytes, uint64_t *b) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(b)) : "memory");
+}
+
 // ------------------------------------------------------------------------- //
 // A1: per-call control reset and label initialisation (Proc. 1 "Init label",
 // "Init actSet", L207)
@@ -459,6 +494,7 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
     __shared__ u64 s_wsum[kWarps];
     static_assert(KW >= 4 && KW <= 32 && (32 % KW) == 0, "rows per warp");
     __shared__ uint32_t s_acts;                           // activations of this CTA (one global atomic)
+    __shared__ uint32_t s_far_cnt[kWarps], s_far_min[kWarps];   // near-far statistics per warp
     Ctl *ctl = d.ctl;
     if (threadIdx.x == 0) s_acts = 0;
     const uint32_t epoch = cld<P>(ctl->epoch) & 0x3FFFFFFFu;
@@ -473,6 +509,28 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
     const uint32_t th = cld<P>(ctl->thresh);              // near-far threshold (SSSP option)
     const bool qmark = !d.nf_delta && (d.tune & kTuneQMark);   // A/B switch: the expand marks Q itself
     const bool stat = !(d.tune & kTuneScanDyn);
+    // Offset staging: a warp with at least d.scan_rows active rows copies its
+    // KW * 32 + 1 row offsets (rounded up to 16 bytes) into shared memory with
+    // ONE bulk copy (cp.async.bulk, completing on the warp's mbarrier), so both
+    // passes read off[v], off[v + 1] from shared memory: one memory round trip
+    // for the warp's whole range instead of one per group of kG rows and pass.
+    // Sparse warps keep the direct loads (a bulk copy moves 4 KB per warp).
+    constexpr uint32_t kOffPad = 16u / (uint32_t)sizeof(OffT);
+    constexpr uint32_t kOffW = (uint32_t)KW * 32u + kOffPad;   // entries per warp buffer (>= KW * 32 + 1)
+    extern __shared__ __align__(128) uint8_t dyn_smem[];
+    OffT *soff = nullptr;
+    uint64_t *sbar = nullptr;
+    uint32_t bphase = 0;
+    const bool can_stage = !P && d.scan_rows != 0;
+    if (can_stage) {
+        soff = reinterpret_cast<OffT *>(dyn_smem) + (size_t)warp * kOffW;
+        sbar = reinterpret_cast<uint64_t *>(dyn_smem + (size_t)kWarps * kOffW * sizeof(OffT)) + warp;
+        if (lane == 0) {
+            mbar_init(sbar, 1);
+            fence_mbar_init();
+        }
+        __syncwarp();
+    }
     for (uint32_t round = 0;; ++round) {
         // first tile = blockIdx.x (CTAs are dispatched in index order, so a
         // tile's predecessors are resident); later tiles from a counter
@@ -549,21 +607,85 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                 wq[j] |= mine;
             }
             if (nf) {
+                // per-warp partials; one atomic pair per tile (below): the
+                // counters are two words every tile updates, so per-warp
+                // atomics would serialise thousands of them on one L2 slice
                 far_cnt = __reduce_add_sync(kFull, far_cnt);
                 far_min = __reduce_min_sync(kFull, far_min);
-                if (lane == 0 && far_cnt) {
-                    atomicAdd(&ctl->far_count, far_cnt);
-                    atomicMin(&ctl->far_min, far_min);
+                if (lane == 0) {
+                    s_far_cnt[warp] = far_cnt;
+                    s_far_min[warp] = far_min;
                 }
-                __threadfence();                          // before this tile publishes
+            }
+        }
+        bool staged = false;
+        // Sparse rows (mid-size active sets: most rows hold one or two active
+        // vertices): the warp lists its active vertices in shared memory (in
+        // vertex order) and walks the list 32 at a time, one vertex per lane,
+        // instead of paying a whole warp step per row.  nlist = list length.
+        uint32_t nlist = 0;
+        bool use_list = false;
+        uint32_t *slist = reinterpret_cast<uint32_t *>(soff);
+        if (can_stage && !qmark) {
+            const uint32_t pc = (uint32_t)__popc(wq[0]);
+            const uint32_t rows = __ballot_sync(kFull, wq[0] != 0u);
+            const uint32_t pincl = warp_incl_scan(pc);
+            nlist = __shfl_sync(kFull, pincl, 31);
+            use_list = nlist && (nlist + 31u) / 32u < (uint32_t)__popc(rows);
+            if (use_list) {
+                __syncwarp();
+                fence_proxy_async();      // earlier async (bulk) writes of the buffer vs these stores
+                uint32_t o = pincl - pc, m = wq[0];
+                while (m) {
+                    const uint32_t b = (uint32_t)(__ffs(m) - 1);
+                    m &= m - 1u;
+                    slist[o++] = (wbase + lane) * 32u + b;
+                }
+                __syncwarp();
+            }
+        }
+        if (can_stage && !use_list) {
+            const uint32_t rows = __ballot_sync(kFull, wq[0] != 0u);
+            if ((uint32_t)__popc(rows) >= d.scan_rows) {
+                staged = true;
+                // an active row holds a vertex < n, so vb < n: at least 2 entries remain
+                const u64 vb = (u64)wbase * 32ull;
+                const u64 avail = (u64)d.n + 1ull - vb;       // entries of off from vb on
+                const uint32_t need = (uint32_t)min((u64)KW * 32ull + 1ull, avail);
+                const uint32_t ncopy = (uint32_t)min((u64)kOffW, avail) & ~(kOffPad - 1u);   // whole 16 B
+                __syncwarp();
+                fence_proxy_async();      // this warp's earlier reads of the buffer before the async write
+                if (ncopy && lane == 0) {
+                    mbar_expect_tx(sbar, ncopy * (uint32_t)sizeof(OffT));
+                    bulk_g2s_plain(soff, d.off + vb, ncopy * (uint32_t)sizeof(OffT), sbar);
+                }
+                for (uint32_t i = ncopy + lane; i < need; i += 32) soff[i] = __ldg(&d.off[vb + i]);   // array end
+                if (ncopy) {
+                    mbar_wait(sbar, bphase);
+                    bphase ^= 1u;
+                }
+                __syncwarp();
             }
         }
         // pass 1: this warp's (kept, shadows); groups of kG words, all offset
         // loads of a group issued before use
         u64 wsum = 0;
         uint32_t nbits = 0;
+        if (use_list) {
+            nbits = nlist;
+            for (uint32_t i0 = 0; i0 < nlist; i0 += 32) {
+                const uint32_t i = i0 + lane;
+                uint32_t c = 0;
+                if (i < nlist) {
+                    const uint32_t v = slist[i];
+                    c = udc_count<UDC>((uint32_t)(__ldg(&d.off[v + 1]) - __ldg(&d.off[v])), d.K, d.K_log2);
+                }
+                const uint32_t kept = __ballot_sync(kFull, c > 0);
+                wsum += ((u64)__popc(kept) << 32) | __reduce_add_sync(kFull, c);
+            }
+        }
 #pragma unroll
-        for (int j = 0; j < 1; ++j) {
+        for (int j = 0; j < (use_list ? 0 : 1); ++j) {
             for (uint32_t k0 = 0; k0 < (uint32_t)KW; k0 += kG) {
                 uint32_t word[kG], any = 0;
 #pragma unroll
@@ -579,8 +701,9 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                     oe[r] = 0;
                     if ((word[r] >> lane) & 1u) {
                         const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
-                        ob[r] = __ldg(&d.off[v]);
-                        oe[r] = __ldg(&d.off[v + 1]);
+                        const uint32_t li = (k0 + r) * 32 + lane;
+                        ob[r] = staged ? soff[li] : __ldg(&d.off[v]);
+                        oe[r] = staged ? soff[li + 1] : __ldg(&d.off[v + 1]);
                     }
                 }
 #pragma unroll
@@ -614,6 +737,19 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
             const uint32_t aggE = (uint32_t)(btotal >> 32), aggS = (uint32_t)btotal;
             uint32_t exclE = 0, exclS = 0;
             if (lane == 0) {
+                if (d.nf_delta && label && !BFSLAB && !qmark) {
+                    // near-far statistics of the tile, visible before its record
+                    uint32_t fc = 0, fm = kInf;
+                    for (int k = 0; k < kWarps; ++k) {
+                        fc += s_far_cnt[k];
+                        fm = min(fm, s_far_min[k]);
+                    }
+                    if (fc) {
+                        atomicAdd(&ctl->far_count, fc);
+                        atomicMin(&ctl->far_min, fm);
+                        __threadfence();
+                    }
+                }
                 const uint32_t fl = tile == 0 ? 2u : 1u;
                 st_volatile_u64(&d.recE[tile], ((u64)aggE << 32) | eb | fl);
                 st_volatile_u64(&d.recS[tile], ((u64)aggS << 32) | eb | fl);
@@ -647,8 +783,36 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
         __syncthreads();
         // pass 2: write the compacted entries, in vertex order, coalesced
         u64 run = s_prefix + wprefix;
+        if (use_list) {
+            for (uint32_t i0 = 0; i0 < nlist; i0 += 32) {
+                const uint32_t i = i0 + lane;
+                uint32_t v = 0, c = 0, dg = 0;
+                OffT ob = 0;
+                if (i < nlist) {
+                    v = slist[i];
+                    ob = __ldg(&d.off[v]);
+                    dg = (uint32_t)(__ldg(&d.off[v + 1]) - ob);
+                    if (BFSLAB) label[v] = new_depth;         // BFS: depth written once, on compaction
+                    c = udc_count<UDC>(dg, d.K, d.K_log2);
+                }
+                const uint32_t kept = __ballot_sync(kFull, c > 0);
+                const uint32_t cincl = __all_sync(kFull, c <= 1u) ? __popc(kept & ((2u << lane) - 1u))
+                                                                  : warp_incl_scan(c);
+                if (c) {
+                    const uint32_t pos = (uint32_t)(run >> 32) + __popc(kept & lt);
+                    const uint32_t sh = (uint32_t)run + cincl - c;
+                    d.F[pos] = v;
+                    d.B[pos] = ob;
+                    d.D[pos] = dg;
+                    d.S[pos] = sh;
+                    if (!BFSLAB && c > 1 && d.snap_used == 2u) d.Lx[pos] = kInf;   // CC: not read yet
+                    for (uint32_t t = (sh + ts - 1) >> tsl; (t << tsl) < sh + c; ++t) d.tile_first[t] = pos;
+                }
+                run += ((u64)__popc(kept) << 32) | __shfl_sync(kFull, cincl, 31);
+            }
+        }
 #pragma unroll
-        for (int j = 0; j < 1; ++j) {
+        for (int j = 0; j < (use_list ? 0 : 1); ++j) {
             for (uint32_t k0 = 0; k0 < (uint32_t)KW; k0 += kG) {
                 uint32_t word[kG], any = 0;
 #pragma unroll
@@ -666,8 +830,9 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                     lv[r] = 0;
                     if ((word[r] >> lane) & 1u) {
                         const uint32_t v = (wbase + 32 * j + k0 + r) * 32 + lane;
-                        ob[r] = __ldg(&d.off[v]);
-                        oe[r] = __ldg(&d.off[v + 1]);
+                        const uint32_t li = (k0 + r) * 32 + lane;
+                        ob[r] = staged ? soff[li] : __ldg(&d.off[v]);
+                        oe[r] = staged ? soff[li + 1] : __ldg(&d.off[v + 1]);
                         if (!BFSLAB && label && qmark) lv[r] = __ldcg(&label[v]);
                     }
                 }
@@ -683,7 +848,10 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                     const uint32_t dg = (uint32_t)(oe[r] - ob[r]);
                     const uint32_t c = bit ? udc_count<UDC>(dg, d.K, d.K_log2) : 0u;
                     const uint32_t kept = __ballot_sync(kFull, c > 0);
-                    const uint32_t cincl = warp_incl_scan(c);
+                    // every vertex of the row <= K edges (the common case): the
+                    // inclusive prefix of c is a popcount
+                    const uint32_t cincl = __all_sync(kFull, c <= 1u) ? __popc(kept & ((2u << lane) - 1u))
+                                                                      : warp_incl_scan(c);
                     if (c) {
                         const uint32_t pos = (uint32_t)(run >> 32) + __popc(kept & lt);
                         const uint32_t sh = (uint32_t)run + cincl - c;
@@ -710,10 +878,12 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
             ctl->tile_ctr = 0;
             ctl->depth = cld<P>(ctl->depth) + 1;
             bool more = nF > 0;
-            if (d.nf_delta && cld<P>(ctl->far_count)) {
+            // (the statistics of other tiles: volatile reads -- this SM's L1 may
+            // hold the control block's line from the kernel start)
+            if (d.nf_delta && cld<true>(ctl->far_count)) {
                 more = true;
                 if (nF == 0) {                        // near set empty: next bucket
-                    const unsigned long long thn = (unsigned long long)cld<P>(ctl->far_min) + d.nf_delta;
+                    const unsigned long long thn = (unsigned long long)cld<true>(ctl->far_min) + d.nf_delta;
                     ctl->thresh = thn > kInf ? kInf : (uint32_t)thn;
                 } else if (!(d.tune & kTuneNearFarClassic)) {   // wave: the threshold advances every iteration
                     const unsigned long long thn = (unsigned long long)th + d.nf_delta;
@@ -729,9 +899,21 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
     if (threadIdx.x == 0 && s_acts) atomicAdd(&ctl->activations, (u64)s_acts);   // result unused: RED
 }
 
+// Programmatic dependent launch (the loop's CUDA graph links expand -> scan
+// with a programmatic edge): a kernel lets its dependent grid launch at once
+// -- the dependent's CTAs take SM slots as this grid's CTAs exit, so there is
+// no launch gap -- and waits for its own primary grid (completion and memory
+// visibility) before touching anything the primary writes.  Without a
+// programmatic edge both instructions are no-ops.
+__device__ __forceinline__ void pdl_begin() {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 template <class OffT, bool UDC, bool BFSLAB, int KW = kWPW>
 __global__ __launch_bounds__(kBlock, 4) void udc_scan_kernel(Dev<OffT> d, cudaGraphConditionalHandle cond,
                                                           int use_cond) {
+    pdl_begin();
     scan_phase<OffT, UDC, BFSLAB, false, KW>(d, cond, use_cond);
 }
 
@@ -1040,33 +1222,6 @@ __device__ __forceinline__ WarpShadow<OffT, UDC> warp_map(const Dev<OffT> &d, ui
     return r;
 }
 
-// ---- mbarrier / bulk-copy helpers (SMP stages) ----
-__device__ __forceinline__ uint32_t smem_u32(const void *p) {
-    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(b)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void fence_mbar_init() {
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(b)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
-    asm volatile("{\n .reg .pred p;\n WAIT_%=:\n"
-                 " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-                 " @!p bra WAIT_%=;\n}" :: "r"(smem_u32(b)), "r"(parity) : "memory");
-}
-__device__ __forceinline__ void fence_proxy_async() {
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
-// TMA bulk copy global -> shared (16-byte aligned, size multiple of 16), completing on mbarrier b
-__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *b, uint64_t pol) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
-                 :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(b)), "l"(pol) : "memory");
-}
-
 // Per-tile state of a warp: its 32 shadows and where their edges live.
 template <class OffT, bool UDC>
 struct WarpTile {
@@ -1075,6 +1230,7 @@ struct WarpTile {
     uint32_t E;        // edges in the tile
     OffT delta;        // element x of this lane's slice is col[delta + x]      (direct)
     uint32_t sdelta;   // ... and stage[sdelta + x] in shared memory            (SMP)
+    uint32_t x0;       // first batch of this warp-unit (tile split: unit / ntiles batches in)
 };
 
 template <class OffT, int ALG, bool UDC, bool SMP, bool P, bool PEER = false>
@@ -1125,7 +1281,19 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
     // The first grab is static (global warp index), later ones come from the
     // counter: a small active set costs no atomic at all, and a large one
     // one atomic per grab after the first.
-    constexpr uint32_t kGrab = 2;
+    // Tile split (sparse iterations): with fewer tiles than warps, G warps share
+    // each tile, warp-unit u taking tile u % ntiles and its batches u / ntiles,
+    // u / ntiles + G, ... -- a hub's edges are not walked by one warp alone.
+    uint32_t G = 1;
+#if ETG_PIPE
+    if (!SMP && !P && d.split && ntiles) {
+        const uint32_t per = (gridDim.x * kWarps) / ntiles;
+        G = per >= 8 ? 8u : per >= 4 ? 4u : per >= 2 ? 2u : 1u;
+        if (G > d.split) G = d.split;
+    }
+#endif
+    const uint32_t nunits = ntiles * G;
+    const uint32_t kGrab = G > 1 ? 1u : 2u;
     const uint32_t n_static = gridDim.x * kWarps * kGrab;
     uint32_t g_next = 0, g_end = 0;
     bool first_grab = true;
@@ -1137,20 +1305,22 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
                 first_grab = false;
             } else {
                 const uint32_t base = ETG_SGRAB ? n_static : 0u;
-                if (lane == 0 && base < ntiles) g = base + atomicAdd(&ctl->tile_ctr, kGrab);
-                g = base < ntiles ? __shfl_sync(kFull, g, 0) : ntiles;
+                if (lane == 0 && base < nunits) g = base + atomicAdd(&ctl->tile_ctr, kGrab);
+                g = base < nunits ? __shfl_sync(kFull, g, 0) : nunits;
             }
             g_next = g;
-            g_end = g_next >= ntiles ? g_next : min(g_next + kGrab, ntiles);
-            if (g_next >= ntiles) return ntiles;
+            g_end = g_next >= nunits ? g_next : min(g_next + kGrab, nunits);
+            if (g_next >= nunits) return nunits;
         }
         return g_next++;
     };
     // Map tile t and start fetching its neighbour segments: SMP -> TMA bulk
     // copies into stage `st` (Sec. V-B: fetch the shadow's neighbours to
     // shared memory before processing them); direct -> L2 bulk prefetch.
-    auto prepare = [&](uint32_t t, uint32_t st) -> WarpTile<OffT, UDC> {
+    auto prepare = [&](uint32_t u, uint32_t st) -> WarpTile<OffT, UDC> {
         WarpTile<OffT, UDC> w;
+        const uint32_t t = G > 1 ? u % ntiles : u;
+        w.x0 = G > 1 ? (u / ntiles) * 32u * (uint32_t)kRB : 0u;
         w.sh = warp_map<OffT, UDC, P>(d, t, nF, N);
         const uint32_t incl = warp_incl_scan(w.sh.len);
         w.o = incl - w.sh.len;
@@ -1212,14 +1382,15 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
     // BFS: live labels; else the snapshot (R-4, R-6), or the live labels when
     // label + snapshot do not fit in L2 (one random stream instead of two)
     const uint32_t *filt = (ALG == ALG_BFS || d.filt_live) ? label : d.snap;
+    const uint32_t xstep = 32u * (uint32_t)kRB * G;       // batch stride of a warp-unit
     uint32_t t = next_tile();
-    if (t < ntiles) {
+    if (t < nunits) {
         WarpTile<OffT, UDC> nxt = prepare(t, 0);
         // stage-A cursor: tile A_t (sequence number kt), batch start A_x0
         WarpTile<OffT, UDC> A_t = nxt;
         uint32_t kt = 0;
         uint32_t tn = next_tile();
-        if (tn < ntiles) nxt = prepare(tn, 1);
+        if (tn < nunits) nxt = prepare(tn, 1);
         // fresh source label (R-6).  Single GPU: a vertex expanded by a sole
         // shadow records the label it propagates in the snapshot, so the scan
         // re-activates it only if its label moves after this read (R-5).
@@ -1233,7 +1404,9 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
             uint32_t l = ld_cg(&label[sh.v]);
             if (snap_used) {
                 if (sh.sole) {
-                    d.snap[sh.v] = l;
+                    // (tile split: the slice may straddle two warps' batches, read
+                    // at different times -- the snapshot keeps the scan-time value)
+                    if (G == 1) d.snap[sh.v] = l;
                 } else if ((ALG == ALG_CC || (ETG_SHARED_SSSP && ALG == ALG_SSSP)) && d.snap_used == 2u) {
 #if ETG_LX_PEEK
                     // published already? (a plain load: hubs of many shadows do not
@@ -1250,19 +1423,21 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
             return l;
         };
         uint32_t A_lab = (ALG == ALG_BFS) ? level : src_label(A_t.sh);
-        uint32_t A_x0 = 0, A_owner = 0xFFFFFFFFu;
+        uint32_t A_x0 = A_t.x0, A_owner = 0xFFFFFFFFu;
         const uint32_t *A_sbuf = nullptr;
         if (SMP) {
             mbar_wait(&bars[0], 0);
             __syncwarp();
             A_sbuf = wbuf;
         }
-        my_edges += A_t.E;
+        if (A_t.x0 == 0) my_edges += A_t.E;
         bool A_valid = true;
         uint32_t u0[kRB], c0[kRB], u1[kRB], c1[kRB];
         uint32_t am0 = 0, am1 = 0;
         // stage A: the batch at (A_t, A_x0) into (u, c, am); then advance the cursor
         auto stage_a = [&](uint32_t (&u)[kRB], uint32_t (&c)[kRB], uint32_t &am) {
+            // owner of the element before the batch (tile split: batches are skipped)
+            if (G > 1) A_owner = (uint32_t)__popc(__ballot_sync(kFull, A_t.sh.len && A_t.o < A_x0)) - 1u;
             const uint32_t pos = A_t.o - A_x0;                 // this lane's slice start in the batch
             const bool in_win = A_t.sh.len && pos < 32u * kRB;
             uint32_t wm[kRB];
@@ -1303,19 +1478,19 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
                 for (int r = 0; r < kRB; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
             }
             // advance: next batch of this tile, or the next tile
-            A_x0 += 32u * kRB;
+            A_x0 += xstep;
             if (A_x0 >= A_t.E) {
-                if (tn >= ntiles) {
+                if (tn >= nunits) {
                     A_valid = false;
                 } else {
                     A_t = nxt;
                     ++kt;
                     tn = next_tile();
-                    if (tn < ntiles) nxt = prepare(tn, (kt + 1) & 1);   // refills the stage of tile kt-1
+                    if (tn < nunits) nxt = prepare(tn, (kt + 1) & 1);   // refills the stage of tile kt-1
                     A_lab = (ALG == ALG_BFS) ? level : src_label(A_t.sh);
-                    A_x0 = 0;
+                    A_x0 = A_t.x0;                             // (>= E: an empty unit, one empty batch)
                     A_owner = 0xFFFFFFFFu;
-                    my_edges += A_t.E;
+                    if (A_t.x0 == 0) my_edges += A_t.E;
                     if (SMP) {
                         mbar_wait(&bars[kt & 1], (kt >> 1) & 1);
                         __syncwarp();
@@ -1497,6 +1672,7 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
 
 template <class OffT, int ALG, bool UDC, bool SMP, bool PEER = false>
 __global__ __launch_bounds__(kBlock, ETG_MINB) void expand_warp_kernel(Dev<OffT> d, uint32_t capw) {
+    pdl_begin();
     expand_phase<OffT, ALG, UDC, SMP, false, PEER>(d, capw);
 }
 
