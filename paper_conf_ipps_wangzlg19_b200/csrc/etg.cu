@@ -166,6 +166,7 @@ struct etg_graph {
     uint32_t scan_smem = 0;               // scan: dynamic shared memory (offset staging buffers + mbarriers)
     uint32_t scan_rows = 0;               // scan: active rows from which a warp stages its offsets (0: never)
     uint32_t split = 8;                   // expand: max warps sharing one tile in sparse iterations (ETG_SPLIT)
+    uint32_t scan_list = 1;               // scan: vertex-list path 0 never, 1 for sparse rows, 2 always (ETG_SCAN_LIST)
     bool pdl = false;                     // loop graph: programmatic expand -> scan edges (ETG_PDL=1; measured
                                           // 1 % slower on C2, per-iteration floor unchanged: off by default)
     int grid_init = 0;
@@ -254,6 +255,7 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     if (own) d.filt_live = 1u;
     d.scan_rows = g->scan_smem ? g->scan_rows : 0u;
     d.split = g->split;
+    d.scan_list = g->scan_list;
     d.npeer = g->npeer;
     d.peer_rank = g->peer_rank;
     for (uint32_t k = 0; k <= kMaxPeer; ++k) d.peer_bounds[k] = g->peer_bounds[k];
@@ -1172,6 +1174,7 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
     // bulk-copies its offsets into shared memory
     if (const char *e_s = getenv("ETG_SPLIT")) g->split = (uint32_t)std::max(1, atoi(e_s));
     if (const char *e_p = getenv("ETG_PDL")) g->pdl = atoi(e_p) != 0;
+    if (const char *e_l = getenv("ETG_SCAN_LIST")) g->scan_list = (uint32_t)atoi(e_l);
     g->scan_rows = 4;
     if (const char *e_r = getenv("ETG_SCAN_ROWS")) g->scan_rows = (uint32_t)atoi(e_r);
     g->scan_smem = 0;

@@ -131,6 +131,7 @@ struct Dev {
     uint32_t snap_used;         // SSSP/CC/SSWP, single GPU: a sole shadow stores the label it expands with
     uint32_t filt_live;         // SSSP/CC/SSWP pre-filter reads the live labels, not the snapshot (label +
                                 // snapshot larger than L2: one randomly gathered array instead of two)
+    uint32_t scan_list;         // scan: vertex-list path 0 never, 1 sparse rows (default), 2 always
     uint32_t split;             // expand: max warps sharing one tile in sparse iterations (1: no split)
     uint32_t scan_rows;         // scan: a warp with >= scan_rows active rows stages its offsets in shared
                                 // memory with one bulk copy (0: never; needs the dynamic shared memory)
@@ -631,7 +632,7 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
             const uint32_t rows = __ballot_sync(kFull, wq[0] != 0u);
             const uint32_t pincl = warp_incl_scan(pc);
             nlist = __shfl_sync(kFull, pincl, 31);
-            use_list = nlist && (nlist + 31u) / 32u < (uint32_t)__popc(rows);
+            use_list = nlist && (d.scan_list == 2u || (d.scan_list == 1u && (nlist + 31u) / 32u < (uint32_t)__popc(rows)));
             if (use_list) {
                 __syncwarp();
                 fence_proxy_async();      // earlier async (bulk) writes of the buffer vs these stores
