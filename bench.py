@@ -199,15 +199,17 @@ def measured_peak():
 
 def ncu_traffic(config, algs):
     """dram bytes per expand launch and the algorithmic bytes of the SAME launches,
-    from the committed ncu summary of this config (profiles/r02/expand_traffic_*.json,
-    tools/traffic_summary.py), if any."""
-    path = os.path.join(ROOT, "profiles", "r02", f"expand_traffic_{config}_{'+'.join(algs)}.json")
-    try:
-        with open(path) as f:
-            d = json.load(f)
-        return d, os.path.relpath(path, ROOT)
-    except (OSError, ValueError):
-        return None, None
+    from the newest committed ncu summary of this config (profiles/r03, else r02:
+    expand_traffic_*.json, tools/traffic_summary.py), if any."""
+    for rnd in ("r03", "r02"):
+        path = os.path.join(ROOT, "profiles", rnd, f"expand_traffic_{config}_{'+'.join(algs)}.json")
+        try:
+            with open(path) as f:
+                d = json.load(f)
+            return d, os.path.relpath(path, ROOT)
+        except (OSError, ValueError):
+            continue
+    return None, None
 
 
 # --------------------------------------------------------------------------- #

@@ -144,6 +144,31 @@ def test_engine_variants(c1, c1sym, monkeypatch, tune):
     check_cc(c1sym, flags=32)
 
 
+@pytest.mark.parametrize("env", [
+    {"ETG_SCAN_LIST": "0"}, {"ETG_SCAN_LIST": "2"}, {"ETG_SCAN_ROWS": "0"}, {"ETG_SCAN_ROWS": "1"},
+    {"ETG_SPLIT": "1"}, {"ETG_SPLIT": "2"}, {"ETG_PDL": "1"}, {"ETG_SCAN_KW": "32", "ETG_SCAN_LIST": "2"}])
+def test_scan_and_split_modes(c1, c1sym, monkeypatch, env):
+    """Load-time scan / expand modes: the vertex-list compaction (never / always),
+    the bulk-copied offsets (off / from one active row), the tile split (off /
+    2 warps), the programmatic expand -> scan edge, 32-row scan tiles on a small
+    graph.  A5 and A2 only reorder how the same active set is compacted and
+    expanded, so labels stay the unique fixpoints; a hub whose
+    shadows span many tiles and the skewed LJ-small shape exercise both paths."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    check_all(c1, gg.sample_sources(c1, 2, 29))
+    check_cc(c1sym)
+    g = gg.make("LJ-small")
+    check_all(g, gg.sample_sources(g, 1, 31), algs=("bfs", "sssp"))
+    off, col, w = g.numpy()
+    s = gg.sample_sources(g, 1, 37)[0]                  # the bench's SSSP schedule (wave, auto Delta)
+    np.testing.assert_array_equal(U32(to_etg(g, sssp_delta="auto").sssp(s)[0]), oracle.sssp(off, col, w, s))
+    n = 200_000
+    hub = [(0, v) for v in range(1, 150_001)] + [(v, v + 1) for v in range(150_000, n - 1)]
+    gh = gg.add_weights(gg.from_edges("hub", n, hub), 7)
+    check_all(gh, [0, 150_000], algs=("bfs", "sssp"))
+
+
 def test_u64_offsets(c1):
     check_all(c1, gg.sample_sources(c1, 2, 3), force_u64=True)
 
