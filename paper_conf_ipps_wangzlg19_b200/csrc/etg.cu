@@ -367,10 +367,12 @@ cudaError_t launch_scan(const etg_graph *g, int alg, void **args, cudaStream_t s
 }
 
 // shared memory of the scan kernels with KW rows per warp: per warp KW * 32 + 1
-// offsets rounded up to 16 bytes, plus one mbarrier
+// offsets rounded up to 16 bytes, one mbarrier, and the vertex list (KW * 32
+// 16-bit indices)
 template <class OffT>
 uint32_t scan_smem_bytes(int kw) {
-    return (uint32_t)(kWarps * ((uint32_t)kw * 32u + 16u / (uint32_t)sizeof(OffT)) * sizeof(OffT) + kWarps * 8);
+    return (uint32_t)(kWarps * ((uint32_t)kw * 32u + 16u / (uint32_t)sizeof(OffT)) * sizeof(OffT) + kWarps * 8 +
+                      kWarps * (uint32_t)kw * 32u * 2u);
 }
 
 // second argument of the expand kernels: CTA kernel -> staging capacity in

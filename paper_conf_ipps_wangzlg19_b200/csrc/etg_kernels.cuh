@@ -520,12 +520,15 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
     constexpr uint32_t kOffW = (uint32_t)KW * 32u + kOffPad;   // entries per warp buffer (>= KW * 32 + 1)
     extern __shared__ __align__(128) uint8_t dyn_smem[];
     OffT *soff = nullptr;
+    uint16_t *slist = nullptr;                               // vertex-list path: row-local vertex indices
     uint64_t *sbar = nullptr;
     uint32_t bphase = 0;
     const bool can_stage = !P && d.scan_rows != 0;
     if (can_stage) {
         soff = reinterpret_cast<OffT *>(dyn_smem) + (size_t)warp * kOffW;
         sbar = reinterpret_cast<uint64_t *>(dyn_smem + (size_t)kWarps * kOffW * sizeof(OffT)) + warp;
+        slist = reinterpret_cast<uint16_t *>(dyn_smem + (size_t)kWarps * (kOffW * sizeof(OffT) + 8u)) +
+                (size_t)warp * KW * 32u;
         if (lane == 0) {
             mbar_init(sbar, 1);
             fence_mbar_init();
@@ -623,10 +626,10 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
         // Sparse rows (mid-size active sets: most rows hold one or two active
         // vertices): the warp lists its active vertices in shared memory (in
         // vertex order) and walks the list 32 at a time, one vertex per lane,
-        // instead of paying a whole warp step per row.  nlist = list length.
+        // instead of paying a whole warp step per row.  nlist = list length;
+        // entries are indices into the warp's 32 * KW vertices.
         uint32_t nlist = 0;
         bool use_list = false;
-        uint32_t *slist = reinterpret_cast<uint32_t *>(soff);
         if (can_stage && !qmark) {
             const uint32_t pc = (uint32_t)__popc(wq[0]);
             const uint32_t rows = __ballot_sync(kFull, wq[0] != 0u);
@@ -634,18 +637,17 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
             nlist = __shfl_sync(kFull, pincl, 31);
             use_list = nlist && (d.scan_list == 2u || (d.scan_list == 1u && (nlist + 31u) / 32u < (uint32_t)__popc(rows)));
             if (use_list) {
-                __syncwarp();
-                fence_proxy_async();      // earlier async (bulk) writes of the buffer vs these stores
+                __syncwarp();             // the previous tile's reads of the list are done
                 uint32_t o = pincl - pc, m = wq[0];
                 while (m) {
                     const uint32_t b = (uint32_t)(__ffs(m) - 1);
                     m &= m - 1u;
-                    slist[o++] = (wbase + lane) * 32u + b;
+                    slist[o++] = (uint16_t)(lane * 32u + b);
                 }
                 __syncwarp();
             }
         }
-        if (can_stage && !use_list) {
+        if (can_stage) {
             const uint32_t rows = __ballot_sync(kFull, wq[0] != 0u);
             if ((uint32_t)__popc(rows) >= d.scan_rows) {
                 staged = true;
@@ -678,8 +680,11 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                 const uint32_t i = i0 + lane;
                 uint32_t c = 0;
                 if (i < nlist) {
-                    const uint32_t v = slist[i];
-                    c = udc_count<UDC>((uint32_t)(__ldg(&d.off[v + 1]) - __ldg(&d.off[v])), d.K, d.K_log2);
+                    const uint32_t li = slist[i];
+                    const uint32_t v = wbase * 32u + li;
+                    const OffT b0 = staged ? soff[li] : __ldg(&d.off[v]);
+                    const OffT b1 = staged ? soff[li + 1] : __ldg(&d.off[v + 1]);
+                    c = udc_count<UDC>((uint32_t)(b1 - b0), d.K, d.K_log2);
                 }
                 const uint32_t kept = __ballot_sync(kFull, c > 0);
                 wsum += ((u64)__popc(kept) << 32) | __reduce_add_sync(kFull, c);
@@ -790,9 +795,10 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                 uint32_t v = 0, c = 0, dg = 0;
                 OffT ob = 0;
                 if (i < nlist) {
-                    v = slist[i];
-                    ob = __ldg(&d.off[v]);
-                    dg = (uint32_t)(__ldg(&d.off[v + 1]) - ob);
+                    const uint32_t li = slist[i];
+                    v = wbase * 32u + li;
+                    ob = staged ? soff[li] : __ldg(&d.off[v]);
+                    dg = (uint32_t)((staged ? soff[li + 1] : __ldg(&d.off[v + 1])) - ob);
                     if (BFSLAB) label[v] = new_depth;         // BFS: depth written once, on compaction
                     c = udc_count<UDC>(dg, d.K, d.K_log2);
                 }
