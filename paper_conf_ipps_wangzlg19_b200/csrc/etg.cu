@@ -166,6 +166,8 @@ struct etg_graph {
     uint32_t scan_smem = 0;               // scan: dynamic shared memory (offset staging buffers + mbarriers)
     uint32_t scan_rows = 0;               // scan: active rows from which a warp stages its offsets (0: never)
     uint32_t split = 8;                   // expand: max warps sharing one tile in sparse iterations (ETG_SPLIT)
+    uint32_t ahead_mid = 1;               // expand: look-ahead in mid-size iterations for every algorithm (ETG_AHEAD_MID)
+    uint32_t tune2 = 0;                   // experiment bits (ETG_TUNE2)
     uint32_t scan_list = 1;               // scan: vertex-list path 0 never, 1 for sparse rows, 2 always (ETG_SCAN_LIST)
     bool pdl = false;                     // loop graph: programmatic expand -> scan edges (ETG_PDL=1; measured
                                           // 1 % slower on C2, per-iteration floor unchanged: off by default)
@@ -256,6 +258,8 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.scan_rows = g->scan_smem ? g->scan_rows : 0u;
     d.split = g->split;
     d.scan_list = g->scan_list;
+    d.ahead_mid = g->p.ahead ? g->ahead_mid : 0u;
+    d.tune2 = g->tune2;
     d.npeer = g->npeer;
     d.peer_rank = g->peer_rank;
     for (uint32_t k = 0; k <= kMaxPeer; ++k) d.peer_bounds[k] = g->peer_bounds[k];
@@ -1177,6 +1181,8 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
     if (const char *e_s = getenv("ETG_SPLIT")) g->split = (uint32_t)std::max(1, atoi(e_s));
     if (const char *e_p = getenv("ETG_PDL")) g->pdl = atoi(e_p) != 0;
     if (const char *e_l = getenv("ETG_SCAN_LIST")) g->scan_list = (uint32_t)atoi(e_l);
+    if (const char *e_a = getenv("ETG_AHEAD_MID")) g->ahead_mid = (uint32_t)atoi(e_a);
+    if (const char *e_t = getenv("ETG_TUNE2")) g->tune2 = (uint32_t)atoi(e_t);
     g->scan_rows = 4;
     if (const char *e_r = getenv("ETG_SCAN_ROWS")) g->scan_rows = (uint32_t)atoi(e_r);
     g->scan_smem = 0;

@@ -127,6 +127,8 @@ struct Dev {
     uint32_t tune;              // experiment switches (ETG_TUNE env var at load); 0 = default
     uint32_t prefetch;          // warp kernel, direct mode: L2 bulk prefetch of the next tile
     uint32_t ahead;             // warp kernel: stage A of the next batch before stage B of this one
+    uint32_t ahead_mid;         // ... also for SSSP/CC/SSWP in mid-size iterations (ETG_AHEAD_MID, default 1)
+    uint32_t tune2;             // experiment bits (ETG_TUNE2): 1 = keep two tiles per grab in mid-size iterations
     uint32_t nf_delta;          // near-far SSSP bucket width (0: the paper's schedule)
     uint32_t snap_used;         // SSSP/CC/SSWP, single GPU: a sole shadow stores the label it expands with
     uint32_t filt_live;         // SSSP/CC/SSWP pre-filter reads the live labels, not the snapshot (label +
@@ -1300,7 +1302,10 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
     }
 #endif
     const uint32_t nunits = ntiles * G;
-    const uint32_t kGrab = G > 1 ? 1u : 2u;
+    // two tiles per grab only when there are plenty (>= 4 per warp): with fewer,
+    // a static grab of two would leave half of the warps without a tile
+    const uint32_t mid = (nunits < 4u * gridDim.x * kWarps) ? 1u : 0u;
+    const uint32_t kGrab = (G > 1 || (mid && (d.tune2 & 1u) == 0)) ? 1u : 2u;
     const uint32_t n_static = gridDim.x * kWarps * kGrab;
     uint32_t g_next = 0, g_end = 0;
     bool first_grab = true;
@@ -1552,7 +1557,10 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
             }
         };
         stage_a(u0, c0, am0);
-        if (!d.ahead) {
+        // look-ahead: d.ahead (BFS), and every algorithm in mid-size
+        // iterations (fewer than 4 tiles per warp: latency-bound, each warp
+        // walks a few batches back to back)
+        if (!(d.ahead || (mid && d.ahead_mid))) {
             // ETG_NO_SMP ("w/o SMP" ablation): each batch's segments are loaded
             // and relaxed back to back, nothing is fetched ahead of its use
             for (;;) {
