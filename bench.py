@@ -212,6 +212,26 @@ def ncu_traffic(config, algs):
     return None, None
 
 
+def l2_roofline(tr, tr_path, avg_launch_ms):
+    """The expand's second roofline: L2 requests from the SMs per second against
+    the chip's measured ceiling for random 4-byte requests (tools/gather_bench.cu,
+    committed as profiles/r03/l2_ceiling.json).  Requests per launch come from the
+    ncu capture of the same launches as `traffic`; the time per launch is this
+    run's CUDA-event mean.  None when either input is missing."""
+    if not tr or not tr.get("l2_requests_per_launch"):
+        return None
+    try:
+        with open(os.path.join(ROOT, "profiles", "r03", "l2_ceiling.json")) as f:
+            ceil = json.load(f)
+    except (OSError, ValueError):
+        return None
+    achieved = tr["l2_requests_per_launch"] / (avg_launch_ms * 1e-3) / 1e9
+    return {"unit": "G requests/s", "achieved": achieved, "ceiling": ceil["ceiling_g_per_s"],
+            "frac": achieved / ceil["ceiling_g_per_s"], "requests_per_launch": tr["l2_requests_per_launch"],
+            "requests_per_edge": tr.get("l2_requests_per_edge"),
+            "source": f"{tr_path} (lts__t_requests_srcunit_tex.sum); ceiling: {ceil['source']}"}
+
+
 # --------------------------------------------------------------------------- #
 # workload
 # --------------------------------------------------------------------------- #
@@ -546,6 +566,7 @@ def run_ours(args):
                 "per_alg": {a: {"achieved_gbs": v["bytes"] / (v["expand_ms"] * 1e-3) / 1e9,
                                 "launches": v["launches"],
                                 "edges_processed": v["edges_processed"]} for a, v in per.items()}}
+        roof["l2"] = l2_roofline(tr, tr_path, exp_ms / max(1, launches_p))
         Gp.close()
         if Gsp:
             Gsp.close()

@@ -31,6 +31,8 @@ def test_bench_line_contract():
     for k in ("bound", "achieved", "peak", "unit", "frac", "traffic"):
         assert k in r, k
     assert 0 < r["frac"] < 1 and r["bound"] == "hbm"
+    if r.get("l2"):                  # the L2-request roofline (committed ncu requests + measured ceiling)
+        assert r["l2"]["achieved"] > 0 and r["l2"]["ceiling"] > 0 and 0 < r["l2"]["frac"] < 2
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     e = d["e2e"]
     assert e["value"] > 0 and e["h2d_bytes_per_step"] > 0 and e["d2h_bytes_per_step"] > 0

@@ -37,4 +37,14 @@ out = {"config": stats["config"], "algs": sorted({c["alg"] for c in stats["calls
        "alg_gbs_under_ncu": alg_bytes / max(us, 1e-9) / 1e3, "dram_gbs_under_ncu": dram / max(us, 1e-9) / 1e3,
        "how": "ncu --cache-control none --clock-control none over every expand launch of one host-loop call per "
               "algorithm (tools/prof_run.py); algorithmic bytes from the same calls' etg_stats"}
+# L2 requests / sectors from the SM side (when the capture has them): the
+# expand's real bound on L2-resident configs is the random-request rate
+req = sum(x.get("lts__t_requests_srcunit_tex.sum", 0) for x in per.values())
+sec = sum(x.get("lts__t_sectors_srcunit_tex.sum", 0) for x in per.values())
+if req:
+    edges = sum(c["edges_processed"] for c in stats["calls"])
+    out.update({"l2_requests_total": req, "l2_sectors_total": sec,
+                "l2_requests_per_launch": req / max(L, 1), "l2_sectors_per_launch": sec / max(L, 1),
+                "l2_requests_per_edge": req / max(edges, 1),
+                "l2_g_requests_per_s_under_ncu": req / max(us, 1e-9) / 1e3})
 print(json.dumps(out, indent=1))
