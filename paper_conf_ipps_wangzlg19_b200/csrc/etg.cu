@@ -223,9 +223,10 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.m = g->m;
     d.prefetch = g->p.prefetch ? 1u : 0u;
     // SMP look-ahead (the next batch's segments loaded while this one relaxes):
-    // BFS only by default -- for SSSP/CC/SSWP the plain batch loop measured
-    // 1-2 % faster on C2 (their kR chunks already keep enough loads in flight)
-    d.ahead = (g->p.ahead && (alg == ALG_BFS || alg < 0 || (g->tune & kTuneAheadAll))) ? 1u : 0u;
+    // BFS, SSSP and SSWP -- the weighted ones since their candidates are formed
+    // in stage B (SSSP C2 1.835 -> 1.79 ms, C3 2.24 -> 2.15 ms); not CC, whose
+    // plain batch loop measured faster (1.232 vs 1.26 ms on C2)
+    d.ahead = (g->p.ahead && (alg != ALG_CC || (g->tune & kTuneAheadAll))) ? 1u : 0u;
     d.K = g->p.K;
     d.K_log2 = 32;
     if (d.K && !(d.K & (d.K - 1))) {

@@ -1444,10 +1444,10 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
         }
         if (A_t.x0 == 0) my_edges += A_t.E;
         bool A_valid = true;
-        uint32_t u0[kRB], c0[kRB], u1[kRB], c1[kRB];
+        uint32_t u0[kRB], c0[kRB], w0[kRB], u1[kRB], c1[kRB], w1[kRB];
         uint32_t am0 = 0, am1 = 0;
         // stage A: the batch at (A_t, A_x0) into (u, c, am); then advance the cursor
-        auto stage_a = [&](uint32_t (&u)[kRB], uint32_t (&c)[kRB], uint32_t &am) {
+        auto stage_a = [&](uint32_t (&u)[kRB], uint32_t (&c)[kRB], uint32_t (&wv)[kRB], uint32_t &am) {
             // owner of the element before the batch (tile split: batches are skipped)
             if (G > 1) A_owner = (uint32_t)__popc(__ballot_sync(kFull, A_t.sh.len && A_t.o < A_x0)) - 1u;
             const uint32_t pos = A_t.o - A_x0;                 // this lane's slice start in the batch
@@ -1457,7 +1457,6 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
             for (int r = 0; r < kRB; ++r)
                 wm[r] = __reduce_or_sync(kFull, (in_win && (pos >> 5) == (uint32_t)r) ? (1u << (pos & 31)) : 0u);
             am = 0;
-            uint32_t wv[kRB];
 #pragma unroll
             for (int r = 0; r < kRB; ++r) {
                 const uint32_t own = A_owner + __popc(wm[r] & lt_eq);
@@ -1485,10 +1484,8 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
                     }
                 }
             }
-            if (kW) {
-#pragma unroll
-                for (int r = 0; r < kRB; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
-            }
+            // (the candidates need the weights: computed in stage B, so the
+            // column and weight loads of this batch stay in flight until then)
             // advance: next batch of this tile, or the next tile
             A_x0 += xstep;
             if (A_x0 >= A_t.E) {
@@ -1512,7 +1509,11 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
             }
         };
         // stage B: pre-filter gathers, then fire-and-forget commits
-        auto stage_b = [&](const uint32_t (&u)[kRB], const uint32_t (&c)[kRB], uint32_t am) {
+        auto stage_b = [&](const uint32_t (&u)[kRB], uint32_t (&c)[kRB], const uint32_t (&wv)[kRB], uint32_t am) {
+            if (kW) {
+#pragma unroll
+                for (int r = 0; r < kRB; ++r) c[r] = candidate<ALG>(c[r], wv[r]);
+            }
             if (d.tune & kTuneNoGather) {                     // replay experiment
                 uint32_t x = 0;
 #pragma unroll
@@ -1556,7 +1557,7 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
                     if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, markQ);
             }
         };
-        stage_a(u0, c0, am0);
+        stage_a(u0, c0, w0, am0);
         // look-ahead: d.ahead (BFS), and every algorithm in mid-size
         // iterations (fewer than 4 tiles per warp: latency-bound, each warp
         // walks a few batches back to back)
@@ -1564,19 +1565,19 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
             // ETG_NO_SMP ("w/o SMP" ablation): each batch's segments are loaded
             // and relaxed back to back, nothing is fetched ahead of its use
             for (;;) {
-                stage_b(u0, c0, am0);
+                stage_b(u0, c0, w0, am0);
                 if (!A_valid) break;
-                stage_a(u0, c0, am0);
+                stage_a(u0, c0, w0, am0);
             }
         } else for (;;) {
             // two named register sets alternate, so no copies between iterations
             const bool more1 = A_valid;
-            if (more1) stage_a(u1, c1, am1);
-            stage_b(u0, c0, am0);
+            if (more1) stage_a(u1, c1, w1, am1);
+            stage_b(u0, c0, w0, am0);
             if (!more1) break;
             const bool more0 = A_valid;
-            if (more0) stage_a(u0, c0, am0);
-            stage_b(u1, c1, am1);
+            if (more0) stage_a(u0, c0, w0, am0);
+            stage_b(u1, c1, w1, am1);
             if (!more0) break;
         }
     }

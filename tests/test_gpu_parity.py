@@ -174,6 +174,16 @@ def test_u64_offsets(c1):
     check_all(c1, gg.sample_sources(c1, 2, 3), force_u64=True)
 
 
+@pytest.mark.parametrize("env", [{}, {"ETG_SCAN_LIST": "2", "ETG_SCAN_ROWS": "1"}, {"ETG_SCAN_LIST": "0"}])
+def test_u64_offsets_scan_paths(monkeypatch, env):
+    """64-bit offsets through the scan's staged-offset and vertex-list paths
+    (8-byte shared-memory offsets, 2 CTAs per SM) on the skewed LJ-small shape."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    g = gg.make("LJ-small")
+    check_all(g, gg.sample_sources(g, 2, 41), algs=("bfs", "sssp"), force_u64=True)
+
+
 @pytest.mark.parametrize("cfg", ["T14", "LJ-small"])
 def test_other_shapes(cfg):
     g = gg.make(cfg)
