@@ -197,12 +197,14 @@ def measured_peak():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def ncu_traffic(config, algs):
+def ncu_traffic(config, algs, flags=0):
     """dram bytes per expand launch and the algorithmic bytes of the SAME launches,
     from the newest committed ncu summary of this config (profiles/r03, else r02:
     expand_traffic_*.json, tools/traffic_summary.py), if any."""
     for rnd in ("r03", "r02"):
-        path = os.path.join(ROOT, "profiles", rnd, f"expand_traffic_{config}_{'+'.join(algs)}.json")
+        # engine flags change the launches (e.g. NO_UDC): their own capture, if any
+        suffix = f"_flags{flags}" if flags else ""
+        path = os.path.join(ROOT, "profiles", rnd, f"expand_traffic_{config}_{'+'.join(algs)}{suffix}.json")
         try:
             with open(path) as f:
                 d = json.load(f)
@@ -543,7 +545,7 @@ def run_ours(args):
                 d["edges_processed"] += st.edges_processed
         peak, peak_src = measured_peak()
         achieved = bytes_tot / (exp_ms * 1e-3) / 1e9
-        tr, tr_path = ncu_traffic(args.config, algs)
+        tr, tr_path = ncu_traffic(args.config, algs, args.flags)
         roof = {"bound": "hbm", "kernel": "expand_warp_kernel", "achieved": achieved, "peak": peak,
                 "unit": "GB/s", "frac": achieved / peak,
                 "traffic": tr["dram_bytes_per_launch"] if tr else None,
