@@ -106,7 +106,7 @@ Params derive(const etg_options *opt, uint32_t tune) {
 }
 
 struct Layout {
-    size_t Q, Lfull, V, snap, F, B, D, S, Lx, tile_first, recE, recS, ctl, total;
+    size_t Q, Lfull, V, snap, F, B, D, S, Lx, tile_first, recE, recS, RD, FR, ctl, total;
     uint32_t nwords;
 };
 
@@ -136,6 +136,8 @@ Layout layout(uint64_t n, uint64_t m, const Params &p) {
     L.tile_first = take(4 * max_tiles);
     L.recE = take(8 * max_scan_tiles);
     L.recS = take(8 * max_scan_tiles);
+    L.RD = take(4ull * ((L.nwords + 31) / 32));      // dirty rows (one bit per 32 vertices)
+    L.FR = take(4ull * ((L.nwords + 31) / 32));      // rows holding deferred (near-far) vertices
     L.ctl = take(sizeof(Ctl));
     L.total = o;
     return L;
@@ -168,6 +170,7 @@ struct etg_graph {
     uint32_t split = 8;                   // expand: max warps sharing one tile in sparse iterations (ETG_SPLIT)
     uint32_t ahead_mid = 1;               // expand: look-ahead in mid-size iterations for every algorithm (ETG_AHEAD_MID)
     uint32_t tune2 = 0;                   // experiment bits (ETG_TUNE2)
+    bool dirty = true;                    // dirty-row scans after sparse expands (ETG_DIRTY=0: off)
     uint32_t scan_list = 1;               // scan: vertex-list path 0 never, 1 for sparse rows, 2 always (ETG_SCAN_LIST)
     bool pdl = false;                     // loop graph: programmatic expand -> scan edges (ETG_PDL=1; measured
                                           // 1 % slower on C2, per-iteration floor unchanged: off by default)
@@ -259,6 +262,9 @@ Dev<OffT> make_dev(const etg_graph *g, int alg = -1) {
     d.scan_rows = g->scan_smem ? g->scan_rows : 0u;
     d.split = g->split;
     d.scan_list = g->scan_list;
+    d.RD = reinterpret_cast<uint32_t *>(g->ws + g->L.RD);
+    d.FR = reinterpret_cast<uint32_t *>(g->ws + g->L.FR);
+    d.dirty_tiles = 0;                        // the fused single-GPU loop only (make_dev_fused)
     d.ahead_mid = g->p.ahead ? g->ahead_mid : 0u;
     d.tune2 = g->tune2;
     d.npeer = g->npeer;
@@ -275,6 +281,10 @@ template <class OffT>
 Dev<OffT> make_dev_fused(const etg_graph *g, int alg) {
     Dev<OffT> d = make_dev<OffT>(g, alg);
     d.npeer = 0;                              // the fused loop is single-partition
+    // dirty rows: SSSP/CC/SSWP with 32-row scan warps; an expand with at most
+    // one tile per warp marks the rows it lowers labels in (ETG_DIRTY=0: off)
+    if (alg != ALG_BFS && g->scan_kw == 32 && g->dirty && !g->comm)
+        d.dirty_tiles = (uint32_t)g->num_sms * 3u * (uint32_t)kWarps;
     // 2 = multi-shadow vertices share one published label too -- CC only:
     // measured 1.48 -> 1.28 ms on C2; SSSP 1.96 -> 2.03 and SSWP 2.13 ->
     // 2.17 (the compare-and-swap round trip per tile costs more than the
@@ -1156,7 +1166,7 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
         (e = cudaEventCreate(&g->pev[2])) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), g->stream)) != cudaSuccess ||
         (e = cudaMemsetAsync(g->ws + L.Q, 0, 4ull * L.nwords, g->stream)) != cudaSuccess ||
-        (e = cudaMemsetAsync(g->ws + L.recE, 0, L.ctl - L.recE, g->stream)) != cudaSuccess) {
+        (e = cudaMemsetAsync(g->ws + L.recE, 0, L.ctl - L.recE, g->stream)) != cudaSuccess) {   // (records, RD, FR)
         return bail(fail(ETG_ECUDA, std::string("load: ") + cudaGetErrorString(e)));
     }
     g->tune = tune;
@@ -1182,6 +1192,7 @@ etg_status etg_load_csr(etg_graph **out, uint64_t n, uint64_t m, const void *d_r
     if (const char *e_s = getenv("ETG_SPLIT")) g->split = (uint32_t)std::max(1, atoi(e_s));
     if (const char *e_p = getenv("ETG_PDL")) g->pdl = atoi(e_p) != 0;
     if (const char *e_l = getenv("ETG_SCAN_LIST")) g->scan_list = (uint32_t)atoi(e_l);
+    if (const char *e_d = getenv("ETG_DIRTY")) g->dirty = atoi(e_d) != 0;
     if (const char *e_a = getenv("ETG_AHEAD_MID")) g->ahead_mid = (uint32_t)atoi(e_a);
     if (const char *e_t = getenv("ETG_TUNE2")) g->tune2 = (uint32_t)atoi(e_t);
     g->scan_rows = 4;

@@ -93,6 +93,7 @@ struct Ctl {
     uint32_t far_min;     //   min label of the deferred (far) marked vertices of the last scan
     uint32_t far_count;   //   number of deferred marked vertices of the last scan
     uint32_t more;        // loop condition computed by the last scan
+    uint32_t rd_valid;    // the last expand marked the rows it lowered labels in (RD): the scan may skip the rest
     uint32_t bar;         // persistent loop: grid-barrier arrivals in the current call
     unsigned long long t_expand_ns;   // persistent loop: %globaltimer time of the expand phases
     unsigned long long t_scan_ns;     //   ... and of the scan phases (block 0's view, barrier to barrier)
@@ -134,6 +135,12 @@ struct Dev {
     uint32_t filt_live;         // SSSP/CC/SSWP pre-filter reads the live labels, not the snapshot (label +
                                 // snapshot larger than L2: one randomly gathered array instead of two)
     uint32_t scan_list;         // scan: vertex-list path 0 never, 1 sparse rows (default), 2 always
+    // Dirty rows (SSSP/CC/SSWP, single GPU, 32-row scan warps): a sparse expand
+    // (<= dirty_tiles tiles) marks the 32-vertex row of every label it lowers in
+    // RD, and the next scan compares label and snapshot only in rows marked in
+    // RD or holding deferred (near-far) vertices, FR; 0 = off.
+    uint32_t dirty_tiles;
+    uint32_t *RD, *FR;          // one bit per row of 32 vertices
     uint32_t split;             // expand: max warps sharing one tile in sparse iterations (1: no split)
     uint32_t scan_rows;         // scan: a warp with >= scan_rows active rows stages its offsets in shared
                                 // memory with one bulk copy (0: never; needs the dynamic shared memory)
@@ -370,6 +377,7 @@ __device__ __forceinline__ void ctl_begin(Ctl *ctl, uint32_t *label, uint32_t so
     ctl->thresh = thresh;         // near-far SSSP: the first threshold (the source has distance 0)
     ctl->far_min = 0xFFFFFFFFu;
     ctl->far_count = 0;
+    ctl->rd_valid = 0;            // the first scan compares every row
     ctl->bar = 0;
     ctl->t_expand_ns = 0;
     ctl->t_scan_ns = 0;
@@ -581,8 +589,53 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
             // Near-far SSSP: a moved vertex at distance >= thresh is deferred
             // -- its snapshot is not refreshed, so it stays "moved" and is
             // looked at again by every later scan until the threshold passes it.
+            // dirty rows (KW == 32: one RD / FR word per warp): after a sparse
+            // expand only the rows it marked and the rows holding deferred
+            // vertices can have label != snapshot
+            const bool use_rows = KW == 32 && d.dirty_tiles && !P;
+            const bool dirty = use_rows && cld<P>(ctl->rd_valid);
+            uint32_t far_rows = 0;
+            if (dirty) {
+                const uint32_t rw = wbase >> 5;
+                uint32_t exm = __ldcg(&d.RD[rw]) | __ldcg(&d.FR[rw]);
+                uint32_t mine = 0;
+                while (exm) {                             // uniform (a word every lane read)
+                    uint32_t rr[2 * kG], lv[2 * kG], sv[2 * kG];
 #pragma unroll
-            for (int j = 0; j < 1; ++j) {
+                    for (int r = 0; r < 2 * kG; ++r) {
+                        rr[r] = exm ? (uint32_t)(__ffs(exm) - 1) : 32u;
+                        exm &= exm - 1u;
+                        const uint32_t v = (wbase + rr[r]) * 32 + lane;
+                        lv[r] = 0;
+                        sv[r] = 0;
+                        if (rr[r] < 32u && v < d.n) {
+                            lv[r] = __ldcg(&label[v]);
+                            sv[r] = __ldcg(&d.snap[v]);
+                        }
+                    }
+#pragma unroll
+                    for (int r = 0; r < 2 * kG; ++r) {
+                        if (rr[r] >= 32u) continue;              // uniform
+                        const bool moved = lv[r] != sv[r];
+                        const bool far = nf && moved && lv[r] >= th;
+                        const uint32_t b = __ballot_sync(kFull, moved && !far);
+                        if (lane == rr[r]) mine = b;
+                        if (moved && !far) d.snap[(wbase + rr[r]) * 32 + lane] = lv[r];   // refresh
+                        if (far) {
+                            ++far_cnt;
+                            far_min = min(far_min, lv[r]);
+                        }
+                        if (__any_sync(kFull, far)) far_rows |= 1u << rr[r];
+                    }
+                }
+                wq[0] |= mine;
+                if (lane == 0) {
+                    d.RD[rw] = 0u;                        // consumed
+                    d.FR[rw] = far_rows;                  // rows examined now: all rows of the word that had any
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < (dirty ? 0 : 1); ++j) {
                 uint32_t mine = 0;
                 for (uint32_t k0 = 0; k0 < (uint32_t)KW; k0 += 2 * kG) {
                     uint32_t lv[2 * kG], sv[2 * kG];
@@ -608,9 +661,14 @@ __device__ __forceinline__ void scan_phase(const Dev<OffT> &d, cudaGraphConditio
                             ++far_cnt;
                             far_min = min(far_min, lv[r]);
                         }
+                        if (use_rows && __any_sync(kFull, far)) far_rows |= 1u << (k0 + r);
                     }
                 }
                 wq[j] |= mine;
+                if (use_rows && lane == 0) {
+                    d.RD[wbase >> 5] = 0u;
+                    d.FR[wbase >> 5] = far_rows;
+                }
             }
             if (nf) {
                 // per-warp partials; one atomic pair per tile (below): the
@@ -1259,8 +1317,11 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
     const uint64_t keep = policy_keep(), stream = policy_stream();
     unsigned long long my_edges = 0;
     uint32_t my_passes = 0;                               // replay experiment counter
+    // dirty rows: a sparse launch marks the rows of the labels it lowers
+    const bool mark_rows = !P && ALG != ALG_BFS && d.dirty_tiles && ntiles <= d.dirty_tiles;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         // bookkeeping for the scan that follows this kernel (stream-ordered)
+        ctl->rd_valid = mark_rows ? 1u : 0u;
         ctl->scan_ctr = 0;
         ctl->epoch = cld<P>(ctl->epoch) + 1;
         ctl->far_min = kInf;
@@ -1554,7 +1615,10 @@ __device__ __forceinline__ void expand_phase(const Dev<OffT> &d, uint32_t capw) 
             } else {
 #pragma unroll
                 for (int r = 0; r < kRB; ++r)
-                    if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) commit<ALG>(label, Q, u[r], c[r], keep, markQ);
+                    if (((am >> r) & 1u) && improves<ALG>(c[r], cur[r])) {
+                        commit<ALG>(label, Q, u[r], c[r], keep, markQ);
+                        if (ALG != ALG_BFS && mark_rows) red_or(&d.RD[u[r] >> 10], 1u << ((u[r] >> 5) & 31u), keep);
+                    }
             }
         };
         stage_a(u0, c0, w0, am0);

@@ -147,12 +147,14 @@ def test_engine_variants(c1, c1sym, monkeypatch, tune):
 @pytest.mark.parametrize("env", [
     {"ETG_SCAN_LIST": "0"}, {"ETG_SCAN_LIST": "2"}, {"ETG_SCAN_ROWS": "0"}, {"ETG_SCAN_ROWS": "1"},
     {"ETG_SPLIT": "1"}, {"ETG_SPLIT": "2"}, {"ETG_PDL": "1"}, {"ETG_SCAN_KW": "32", "ETG_SCAN_LIST": "2"},
-    {"ETG_AHEAD_MID": "0", "ETG_TUNE2": "1"}])
+    {"ETG_AHEAD_MID": "0", "ETG_TUNE2": "1"}, {"ETG_DIRTY": "0"}, {"ETG_SCAN_KW": "32"},
+    {"ETG_SCAN_KW": "32", "ETG_SCAN_LIST": "0"}])
 def test_scan_and_split_modes(c1, c1sym, monkeypatch, env):
     """Load-time scan / expand modes: the vertex-list compaction (never / always),
     the bulk-copied offsets (off / from one active row), the tile split (off /
     2 warps), the programmatic expand -> scan edge, 32-row scan tiles on a small
-    graph, the mid-size look-ahead and grab size.  A5 and A2 only reorder how the same active set is compacted and
+    graph, the mid-size look-ahead and grab size, the dirty-row scans (which
+    need 32-row scan warps: forced on the small graphs here).  A5 and A2 only reorder how the same active set is compacted and
     expanded, so labels stay the unique fixpoints; a hub whose
     shadows span many tiles and the skewed LJ-small shape exercise both paths."""
     for k, v in env.items():
