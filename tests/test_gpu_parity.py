@@ -388,13 +388,18 @@ def test_galois_gr_file_traversal(tmp_path, c1):
     np.testing.assert_array_equal(U32(G.sssp(s)[0]), oracle.sssp(off, col, w, s))
 
 
+@pytest.mark.parametrize("rows32", [False, True])
 @pytest.mark.parametrize("classic", [False, True])
 @pytest.mark.parametrize("delta", [3, 12, 40])
-def test_sssp_wave_and_classic_near_far(c1, delta, classic, monkeypatch):
+def test_sssp_wave_and_classic_near_far(c1, delta, classic, rows32, monkeypatch):
     """Both threshold rules of the near-far schedule: the wave (default: the
     threshold advances by Delta every iteration) and the classic one (advance
-    only when the near set is empty; ETG_TUNE=8192).  Same distances."""
+    only when the near set is empty; ETG_TUNE=8192).  Same distances.  rows32:
+    32-row scan warps, so the dirty-row scans (rows marked by the sparse
+    expands plus rows holding deferred vertices) run on these small graphs too."""
     monkeypatch.setenv("ETG_TUNE", "8192" if classic else "0")
+    if rows32:
+        monkeypatch.setenv("ETG_SCAN_KW", "32")
     off, col, w = c1.numpy()
     for s in gg.sample_sources(c1, 2, 100 + delta):
         G = to_etg(c1, sssp_delta=delta)
